@@ -1,0 +1,179 @@
+"""B200-native FEVES inter-prediction hot path: FSBM ME -> INT -> SME.
+
+Thin ctypes binding over ``libfeves_me.so`` (C-ABI in include/feves_me.h).
+Argument marshalling only: every arithmetic step runs in the sm_100a kernels
+of ``csrc/``.  PyTorch provides device memory and streams.  There is no CPU
+fallback: if the library or a CUDA device is missing, every call raises.
+
+Paper: Ilic, Momcilovic, Roma, Sousa, "FEVES: Framework for Efficient Parallel
+Video Encoding on Heterogeneous Systems", ICPP 2014 (/root/reference/PAPER.md,
+P:6 defines ME/INT/SME; P:51 the MB-row distributions used by ``shard``).
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import torch
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libfeves_me.so")
+N_PART = 41
+N_PHASE = 16
+
+ME_OK, ME_EINVAL, ME_ENOMEM, ME_ECUDA, ME_ESTATE = 0, -1, -2, -3, -4
+
+_lib = None
+
+
+class FevesError(RuntimeError):
+    pass
+
+
+def lib():
+    """Load libfeves_me.so (built in-tree by __graft_entry__.build())."""
+    global _lib
+    if _lib is None:
+        if not os.path.exists(LIB_PATH):
+            raise FevesError(f"{LIB_PATH} missing: run `python -c 'import __graft_entry__ as g; g.build()'`")
+        L = ctypes.CDLL(LIB_PATH)
+        P, i = ctypes.c_void_p, ctypes.c_int
+        L.me_create.restype = P
+        L.me_create.argtypes = [i, i, i, i]
+        L.me_destroy.argtypes = [P]
+        L.me_last_error.restype = i
+        L.me_strerror.restype = ctypes.c_char_p
+        L.me_strerror.argtypes = [i]
+        L.me_set_stream.argtypes = [P, P]
+        L.me_set_rows.argtypes = [P, i, i]
+        L.me_get_layout.argtypes = [P, P, P, P, P, P]
+        L.me_estimate.argtypes = [P, P, P, P, P]
+        L.int_interpolate.argtypes = [P, P, P]
+        L.sme_refine.argtypes = [P, P, P, P, P, P, P]
+        L.me_encode_frame.argtypes = [P, P, P, P, i, P, P, P, P]
+        L.me_last_launch_count.argtypes = [P]
+        for fn in ("me_set_stream", "me_set_rows", "me_get_layout", "me_estimate", "int_interpolate",
+                   "sme_refine", "me_encode_frame", "me_last_launch_count"):
+            getattr(L, fn).restype = i
+        _lib = L
+    return _lib
+
+
+def _check(rc):
+    if rc != ME_OK:
+        raise FevesError(f"libfeves_me: {lib().me_strerror(rc).decode()} ({rc})")
+
+
+def _dev_u8(t, name):
+    if not (isinstance(t, torch.Tensor) and t.is_cuda and t.dtype == torch.uint8 and t.is_contiguous()):
+        raise FevesError(f"{name}: expected a contiguous uint8 CUDA tensor")
+    return t
+
+
+def _ptrs(ts):
+    return (ctypes.c_void_p * len(ts))(*[t.data_ptr() for t in ts])
+
+
+class MotionEstimator:
+    """One libfeves_me context: W x H frames, SA side ``sa_range``, ``n_rf`` RFs.
+
+    MV/SAD tensors have shape [rows, mb_cols, n_rf, 41, 2] int16 and
+    [rows, mb_cols, n_rf, 41] uint16 (rows = the current MB-row stripe).
+    """
+
+    def __init__(self, width: int, height: int, sa_range: int, n_rf: int, device=None):
+        if not torch.cuda.is_available():
+            raise FevesError("no CUDA device: the FEVES path has no CPU fallback")
+        self.device = torch.device("cuda", torch.cuda.current_device() if device is None else
+                                   torch.device(device).index or 0)
+        with torch.cuda.device(self.device):
+            L = lib()
+            self._ctx = L.me_create(width, height, sa_range, n_rf)
+            if not self._ctx:
+                raise FevesError(f"me_create({width},{height},{sa_range},{n_rf}): "
+                                 f"{L.me_strerror(L.me_last_error()).decode()}")
+        self.width, self.height, self.sa_range, self.n_rf = width, height, sa_range, n_rf
+        vals = [ctypes.c_int() for _ in range(5)]
+        _check(lib().me_get_layout(self._ctx, *[ctypes.byref(v) for v in vals]))
+        self.mb_cols, self.mb_rows, self.sf_pad, self.sf_pitch, self.sf_rows = [v.value for v in vals]
+        self.row0, self.row1 = 0, self.mb_rows
+
+    def close(self):
+        if getattr(self, "_ctx", None):
+            lib().me_destroy(self._ctx)
+            self._ctx = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    # ------------------------------------------------------------ config --
+    def set_rows(self, r0: int, r1: int):
+        _check(lib().me_set_rows(self._ctx, r0, r1))
+        self.row0, self.row1 = r0, r1
+
+    def _bind_stream(self):
+        _check(lib().me_set_stream(self._ctx, ctypes.c_void_p(torch.cuda.current_stream(self.device).cuda_stream)))
+
+    @property
+    def launches(self) -> int:
+        return lib().me_last_launch_count(self._ctx)
+
+    def mv_shape(self):
+        return (self.row1 - self.row0, self.mb_cols, self.n_rf, N_PART)
+
+    def sf_shape(self):
+        return (N_PHASE, self.sf_rows, self.sf_pitch)
+
+    def new_mvs(self):
+        return (torch.empty(self.mv_shape() + (2,), dtype=torch.int16, device=self.device),
+                torch.empty(self.mv_shape(), dtype=torch.uint16, device=self.device))
+
+    def new_sf(self):
+        return torch.empty(self.sf_shape(), dtype=torch.uint8, device=self.device)
+
+    # ------------------------------------------------------------- calls --
+    def estimate(self, cf, rfs, out=None):
+        """Integer FSBM ME (me_estimate).  Returns (mvs, sads)."""
+        _dev_u8(cf, "cf")
+        assert len(rfs) == self.n_rf
+        for r in rfs:
+            _dev_u8(r, "rf")
+        mvs, sads = out if out is not None else self.new_mvs()
+        self._bind_stream()
+        _check(lib().me_estimate(self._ctx, cf.data_ptr(), _ptrs(rfs), mvs.data_ptr(), sads.data_ptr()))
+        return mvs, sads
+
+    def interpolate(self, rf, out=None):
+        """INT (int_interpolate): 16 phase planes [16, sf_rows, sf_pitch] u8."""
+        _dev_u8(rf, "rf")
+        sf = self.new_sf() if out is None else out
+        self._bind_stream()
+        _check(lib().int_interpolate(self._ctx, rf.data_ptr(), sf.data_ptr()))
+        return sf
+
+    def refine(self, cf, sfs, mvs, sads=None, out=None):
+        """SME (sme_refine).  Returns (qmvs quarter-pel, sads)."""
+        _dev_u8(cf, "cf")
+        assert len(sfs) == self.n_rf
+        qmvs, qsads = out if out is not None else self.new_mvs()
+        self._bind_stream()
+        _check(lib().sme_refine(self._ctx, cf.data_ptr(), _ptrs(sfs), mvs.data_ptr(),
+                                None if sads is None else sads.data_ptr(), qmvs.data_ptr(), qsads.data_ptr()))
+        return qmvs, qsads
+
+    def encode_frame(self, cf, rfs, sfs, n_int, out_me=None, out_sme=None):
+        """INT (first n_int RFs) -> ME -> SME in one C call (me_encode_frame)."""
+        qmvs, qsads = out_sme if out_sme is not None else self.new_mvs()
+        mvs, sads = out_me if out_me is not None else (None, None)
+        self._bind_stream()
+        _check(lib().me_encode_frame(self._ctx, cf.data_ptr(), _ptrs(rfs), _ptrs(sfs), n_int,
+                                     None if mvs is None else mvs.data_ptr(),
+                                     None if sads is None else sads.data_ptr(),
+                                     qmvs.data_ptr(), qsads.data_ptr()))
+        return (mvs, sads), (qmvs, qsads)
+
+
+__all__ = ["MotionEstimator", "FevesError", "lib", "LIB_PATH", "N_PART", "N_PHASE"]

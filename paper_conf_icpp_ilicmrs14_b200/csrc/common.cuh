@@ -1,0 +1,42 @@
+// common.cuh -- small device helpers shared by the sm_100a kernels of
+// libfeves_me.so.  (Product code: never shared with oracle/.)
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace feves {
+
+constexpr int kNPart = 41;     // partitions of the 7 modes (P:6), order G7
+constexpr int kMaxRf = 16;
+
+// d = c + sum_{i<4} |a.byte_i - b.byte_i|  -> one VABSDIFF4.U8.ACC (SURVEY §2.7,
+// verified in SASS; the intrinsic __vsadu4 does not chain the accumulator).
+__device__ __forceinline__ uint32_t vad4(uint32_t a, uint32_t b, uint32_t c) {
+  uint32_t d;
+  asm("vabsdiff4.u32.u32.u32.add %0, %1, %2, %3;" : "=r"(d) : "r"(a), "r"(b), "r"(c));
+  return d;
+}
+
+// per-byte rounded average (u+v+1)>>1 on 4 packed bytes (VAVRG4)
+__device__ __forceinline__ uint32_t vavg4(uint32_t a, uint32_t b) {
+  uint32_t d;
+  asm("vavrg4.u32.u32.u32 %0, %1, %2, %3;" : "=r"(d) : "r"(a), "r"(b), "r"(0u));
+  return d;
+}
+
+__device__ __forceinline__ int clampi(int v, int lo, int hi) { return v < lo ? lo : (v > hi ? hi : v); }
+
+// Four bytes of row y of a W x H tight u8 frame starting at column x, with
+// coordinate clamping (G5).  Fast path: one aligned 32-bit load.
+__device__ __forceinline__ uint32_t load4_clamped(const uint8_t* __restrict__ f, int W, int H, int x, int y) {
+  y = clampi(y, 0, H - 1);
+  const uint8_t* row = f + (size_t)y * W;
+  if (x >= 0 && x + 3 < W && ((reinterpret_cast<uintptr_t>(row + x) & 3) == 0))
+    return __ldg(reinterpret_cast<const uint32_t*>(row + x));
+  uint32_t v = 0;
+#pragma unroll
+  for (int i = 0; i < 4; ++i) v |= (uint32_t)__ldg(row + clampi(x + i, 0, W - 1)) << (8 * i);
+  return v;
+}
+
+}  // namespace feves

@@ -1,0 +1,284 @@
+// feves_me.cu -- libfeves_me.so: the C-ABI of include/feves_me.h over the
+// sm_100a kernels (me_fsbm.cuh, int_subpel.cuh, sme_refine.cuh).
+//
+// The context owns: the spiral-rank tables of G4 (built here with the CLOSED
+// FORM; the oracle enumerates the spiral independently), ME scratch for
+// me_encode_frame, and its stream.  No allocation on the per-frame path.
+#include "../../include/feves_me.h"
+
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <mutex>
+#include <vector>
+
+#include "int_subpel.cuh"
+#include "me_fsbm.cuh"
+#include "sme_refine.cuh"
+
+using namespace feves;
+
+struct me_ctx {
+  int W, H, S, R, n_rf;
+  int mb_cols, mb_rows, row0, row1;
+  int sf_pad, sf_pitch, sf_rows;
+  int device;
+  cudaStream_t stream;
+  bool own_stream;
+  uint32_t* d_rank;      // [S][S]
+  uint32_t* d_inv;       // [(S+1)^2]
+  int16_t* d_mvs;        // scratch for me_encode_frame (full frame)
+  uint16_t* d_sads;
+  // ME launch geometry
+  int lx, ngx, nsub, nwy, dyl, pw, cstride, me_threads;
+  size_t me_smem;
+  int last_launches;
+  const void* checked[64];
+  int n_checked;
+};
+
+static thread_local int g_last_error = ME_OK;
+
+// ------------------------------------------------------------- helpers ----
+static int spiral_rank_closed_form(int dx, int dy) {   // G4
+  const int l = std::max(std::abs(dx), std::abs(dy));
+  if (l == 0) return 0;
+  const int base = (2 * l - 1) * (2 * l - 1);
+  if (std::abs(dy) == l && std::abs(dx) < l) return base + 2 * (dx + l - 1) + (dy > 0 ? 1 : 0);
+  return base + 2 * (2 * l - 1) + 2 * (dy + l) + (dx > 0 ? 1 : 0);
+}
+
+static bool is_device_ptr(me_ctx* c, const void* p) {
+  if (!p) return false;
+  for (int i = 0; i < c->n_checked; ++i)
+    if (c->checked[i] == p) return true;
+  cudaPointerAttributes a;
+  if (cudaPointerGetAttributes(&a, p) != cudaSuccess) { cudaGetLastError(); return false; }
+  if (!(a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged) || a.device != c->device) return false;
+  c->checked[c->n_checked % 64] = p;
+  if (c->n_checked < 64) c->n_checked++;
+  return true;
+}
+
+static int launch_status() {
+  const cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) { fprintf(stderr, "feves_me: %s\n", cudaGetErrorString(e)); return ME_ECUDA; }
+  return ME_OK;
+}
+
+// ------------------------------------------------------------ lifetime ----
+extern "C" me_ctx* me_create(int width, int height, int sa_range, int n_rf) {
+  g_last_error = ME_EINVAL;
+  if (width <= 0 || height <= 0 || width > 16384 || height > 16384) return nullptr;
+  if (sa_range < 4 || sa_range > 128 || (sa_range & 1)) return nullptr;
+  if (n_rf < 1 || n_rf > kMaxRf) return nullptr;
+  me_ctx* c = new (std::nothrow) me_ctx();
+  if (!c) { g_last_error = ME_ENOMEM; return nullptr; }
+  c->W = width; c->H = height; c->S = sa_range; c->R = sa_range / 2; c->n_rf = n_rf;
+  c->mb_cols = (width + 15) / 16; c->mb_rows = (height + 15) / 16;
+  c->row0 = 0; c->row1 = c->mb_rows;
+  c->sf_pad = ((c->R + 4 + 15) / 16) * 16;
+  c->sf_pitch = 16 * c->mb_cols + 2 * c->sf_pad;
+  c->sf_rows = 16 * c->mb_rows + 2 * c->sf_pad;
+  if (cudaGetDevice(&c->device) != cudaSuccess) { delete c; g_last_error = ME_ECUDA; return nullptr; }
+
+  // lane geometry (me_fsbm.cuh): 32 dx per warp (fewer lanes per dx group for
+  // small SAs, the rest of the warp takes other dy sub-ranges)
+  const int S = c->S;
+  c->lx = S >= 32 ? 32 : S >= 16 ? 16 : S >= 8 ? 8 : 4;
+  c->ngx = (S + c->lx - 1) / c->lx;
+  c->nsub = 32 / c->lx;
+  c->nwy = 1;
+  const int parts = c->nsub * c->nwy;
+  c->dyl = ((S + parts - 1) / parts + kMeT - 1) / kMeT * kMeT;
+  c->pw = ((S - 1) >> 2) + 4;
+  const int words = (S + 15) * c->pw;
+  c->cstride = words + ((8 - words % 32) % 32 + 32) % 32;       // cstride = 8 (mod 32): conflict-free copies
+  c->me_threads = 32 * c->ngx * c->nwy;
+  c->me_smem = (size_t)(4 * c->cstride + (c->me_threads / 32) * kNPart) * 4;
+
+  std::vector<uint32_t> rank((size_t)S * S), inv((size_t)(S + 1) * (S + 1), 0);
+  for (int dy = -c->R; dy < c->R; ++dy)
+    for (int dx = -c->R; dx < c->R; ++dx) {
+      const int r = spiral_rank_closed_form(dx, dy);
+      rank[(size_t)(dy + c->R) * S + (dx + c->R)] = (uint32_t)r;
+      inv[r] = (uint32_t)(uint16_t)dx | ((uint32_t)(uint16_t)dy << 16);
+    }
+  const size_t nmv = (size_t)c->mb_cols * c->mb_rows * n_rf * kNPart;
+  bool ok = cudaMalloc(&c->d_rank, rank.size() * 4) == cudaSuccess &&
+            cudaMalloc(&c->d_inv, inv.size() * 4) == cudaSuccess &&
+            cudaMalloc(&c->d_mvs, nmv * 4) == cudaSuccess &&
+            cudaMalloc(&c->d_sads, nmv * 2) == cudaSuccess &&
+            cudaStreamCreateWithFlags(&c->stream, cudaStreamNonBlocking) == cudaSuccess;
+  if (ok) {
+    c->own_stream = true;
+    ok = cudaMemcpy(c->d_rank, rank.data(), rank.size() * 4, cudaMemcpyHostToDevice) == cudaSuccess &&
+         cudaMemcpy(c->d_inv, inv.data(), inv.size() * 4, cudaMemcpyHostToDevice) == cudaSuccess &&
+         cudaFuncSetAttribute(me_fsbm_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                              (int)c->me_smem) == cudaSuccess;
+  }
+  if (!ok) {
+    cudaGetLastError();
+    me_destroy(c);
+    g_last_error = ME_ENOMEM;
+    return nullptr;
+  }
+  g_last_error = ME_OK;
+  return c;
+}
+
+extern "C" void me_destroy(me_ctx* c) {
+  if (!c) return;
+  if (c->own_stream && c->stream) cudaStreamSynchronize(c->stream);
+  cudaFree(c->d_rank);
+  cudaFree(c->d_inv);
+  cudaFree(c->d_mvs);
+  cudaFree(c->d_sads);
+  if (c->own_stream && c->stream) cudaStreamDestroy(c->stream);
+  delete c;
+}
+
+extern "C" int me_last_error(void) { return g_last_error; }
+
+extern "C" const char* me_strerror(int s) {
+  switch (s) {
+    case ME_OK: return "ok";
+    case ME_EINVAL: return "invalid argument";
+    case ME_ENOMEM: return "out of memory";
+    case ME_ECUDA: return "CUDA error";
+    case ME_ESTATE: return "bad context state";
+    default: return "unknown status";
+  }
+}
+
+extern "C" int me_set_stream(me_ctx* c, void* s) {
+  if (!c) return ME_EINVAL;
+  if (c->own_stream && c->stream) { cudaStreamSynchronize(c->stream); cudaStreamDestroy(c->stream); }
+  c->own_stream = false;
+  c->stream = (cudaStream_t)s;
+  return ME_OK;
+}
+
+extern "C" int me_set_rows(me_ctx* c, int r0, int r1) {
+  if (!c || r0 < 0 || r1 > c->mb_rows || r0 >= r1) return ME_EINVAL;
+  c->row0 = r0; c->row1 = r1;
+  return ME_OK;
+}
+
+extern "C" int me_get_layout(const me_ctx* c, int* mb_cols, int* mb_rows, int* sf_pad, int* sf_pitch,
+                             int* sf_rows) {
+  if (!c) return ME_EINVAL;
+  if (mb_cols) *mb_cols = c->mb_cols;
+  if (mb_rows) *mb_rows = c->mb_rows;
+  if (sf_pad) *sf_pad = c->sf_pad;
+  if (sf_pitch) *sf_pitch = c->sf_pitch;
+  if (sf_rows) *sf_rows = c->sf_rows;
+  return ME_OK;
+}
+
+extern "C" int me_last_launch_count(const me_ctx* c) { return c ? c->last_launches : -1; }
+
+// --------------------------------------------------------------- launches ----
+static int launch_me(me_ctx* c, const uint8_t* cf, const uint8_t* const* rfs, int16_t* mvs, uint16_t* sads) {
+  MeParams P;
+  memset(&P, 0, sizeof(P));
+  P.cf = cf;
+  for (int k = 0; k < c->n_rf; ++k) P.rf[k] = rfs[k];
+  P.W = c->W; P.H = c->H; P.S = c->S; P.R = c->R; P.n_rf = c->n_rf;
+  P.mb_cols = c->mb_cols; P.row0 = c->row0;
+  P.rank_tab = c->d_rank; P.inv_tab = c->d_inv;
+  P.out_mvs = mvs; P.out_sads = sads;
+  P.lx = c->lx; P.ngx = c->ngx; P.nsub = c->nsub; P.nwy = c->nwy; P.dyl = c->dyl;
+  P.pw = c->pw; P.cstride = c->cstride;
+  dim3 grid(c->mb_cols, c->row1 - c->row0);
+  me_fsbm_kernel<<<grid, c->me_threads, c->me_smem, c->stream>>>(P);
+  c->last_launches++;
+  return launch_status();
+}
+
+static int launch_int(me_ctx* c, const uint8_t* rf, uint8_t* sf) {
+  IntParams P;
+  P.rf = rf; P.sf = sf; P.W = c->W; P.H = c->H;
+  P.pad = c->sf_pad; P.pitch = c->sf_pitch; P.rows = c->sf_rows;
+  P.plane = (size_t)c->sf_rows * c->sf_pitch;
+  if (c->row0 == 0 && c->row1 == c->mb_rows) {
+    P.row_begin = 0; P.row_end = c->sf_rows;
+  } else {   // stripe + halo: SME reads integer rows [16r0-R-1, 16r1+R-2]
+    P.row_begin = std::max(0, c->sf_pad + 16 * c->row0 - c->R - 4);
+    P.row_end = std::min(c->sf_rows, c->sf_pad + 16 * c->row1 + c->R + 4);
+  }
+  const int groups = c->sf_pitch / 16;
+  dim3 block(32, 4);
+  dim3 grid((groups + 31) / 32, (P.row_end - P.row_begin + 3) / 4);
+  int_subpel_kernel<<<grid, block, 0, c->stream>>>(P);
+  c->last_launches++;
+  return launch_status();
+}
+
+static int launch_sme(me_ctx* c, const uint8_t* cf, const uint8_t* const* sfs, const int16_t* in_mvs,
+                      const uint16_t* in_sads, int16_t* out_qmvs, uint16_t* out_sads) {
+  SmeParams P;
+  memset(&P, 0, sizeof(P));
+  P.cf = cf;
+  for (int k = 0; k < c->n_rf; ++k) P.sf[k] = sfs[k];
+  P.in_mvs = reinterpret_cast<const uint32_t*>(in_mvs);
+  P.in_sads = in_sads;
+  P.out_qmvs = reinterpret_cast<uint32_t*>(out_qmvs);
+  P.out_sads = out_sads;
+  P.W = c->W; P.H = c->H; P.n_rf = c->n_rf; P.mb_cols = c->mb_cols; P.row0 = c->row0;
+  P.n_items = (c->row1 - c->row0) * c->mb_cols * c->n_rf;
+  P.pad = c->sf_pad; P.pitch = c->sf_pitch;
+  P.plane = (size_t)c->sf_rows * c->sf_pitch;
+  const int per_block = 128 / 16;
+  sme_refine_kernel<<<(P.n_items + per_block - 1) / per_block, 128, 0, c->stream>>>(P);
+  c->last_launches++;
+  return launch_status();
+}
+
+// ------------------------------------------------------------------ API ----
+extern "C" int me_estimate(me_ctx* c, const uint8_t* cf, const uint8_t* const* rfs, int16_t* out_mvs,
+                           uint16_t* out_sads) {
+  if (!c || !rfs) return ME_EINVAL;
+  if (!is_device_ptr(c, cf) || !is_device_ptr(c, out_mvs) || !is_device_ptr(c, out_sads)) return ME_EINVAL;
+  for (int k = 0; k < c->n_rf; ++k)
+    if (!is_device_ptr(c, rfs[k])) return ME_EINVAL;
+  c->last_launches = 0;
+  return launch_me(c, cf, rfs, out_mvs, out_sads);
+}
+
+extern "C" int int_interpolate(me_ctx* c, const uint8_t* rf, uint8_t* out_sf) {
+  if (!c || !is_device_ptr(c, rf) || !is_device_ptr(c, out_sf)) return ME_EINVAL;
+  c->last_launches = 0;
+  return launch_int(c, rf, out_sf);
+}
+
+extern "C" int sme_refine(me_ctx* c, const uint8_t* cf, const uint8_t* const* sfs, const int16_t* in_mvs,
+                          const uint16_t* in_sads, int16_t* out_qmvs, uint16_t* out_sads) {
+  if (!c || !sfs) return ME_EINVAL;
+  if (!is_device_ptr(c, cf) || !is_device_ptr(c, in_mvs) || !is_device_ptr(c, out_qmvs) ||
+      !is_device_ptr(c, out_sads))
+    return ME_EINVAL;
+  if (in_sads && !is_device_ptr(c, in_sads)) return ME_EINVAL;
+  for (int k = 0; k < c->n_rf; ++k)
+    if (!is_device_ptr(c, sfs[k])) return ME_EINVAL;
+  c->last_launches = 0;
+  return launch_sme(c, cf, sfs, in_mvs, in_sads, out_qmvs, out_sads);
+}
+
+extern "C" int me_encode_frame(me_ctx* c, const uint8_t* cf, const uint8_t* const* rfs, uint8_t* const* sfs,
+                               int n_int, int16_t* out_mvs, uint16_t* out_sads, int16_t* out_qmvs,
+                               uint16_t* out_qsads) {
+  if (!c || !rfs || !sfs || n_int < 0 || n_int > c->n_rf) return ME_EINVAL;
+  if (!is_device_ptr(c, cf) || !is_device_ptr(c, out_qmvs) || !is_device_ptr(c, out_qsads)) return ME_EINVAL;
+  if ((out_mvs && !is_device_ptr(c, out_mvs)) || (out_sads && !is_device_ptr(c, out_sads))) return ME_EINVAL;
+  for (int k = 0; k < c->n_rf; ++k)
+    if (!is_device_ptr(c, rfs[k]) || !is_device_ptr(c, sfs[k])) return ME_EINVAL;
+  int16_t* mvs = out_mvs ? out_mvs : c->d_mvs;
+  uint16_t* sads = out_sads ? out_sads : c->d_sads;
+  c->last_launches = 0;
+  int st;
+  for (int k = 0; k < n_int; ++k)
+    if ((st = launch_int(c, rfs[k], sfs[k])) != ME_OK) return st;
+  if ((st = launch_me(c, cf, rfs, mvs, sads)) != ME_OK) return st;
+  return launch_sme(c, cf, reinterpret_cast<const uint8_t* const*>(sfs), mvs, sads, out_qmvs, out_qsads);
+}

@@ -1,0 +1,235 @@
+"""GPU parity: the CUDA path (through the C-ABI) vs the CPU oracle, element by element.
+
+Bar: bit-exact (all arithmetic on the path is integer).  MVs are unique under
+G4/G14, so MVs and SADs are compared exactly.  Small cases run the oracle on
+the whole frame (several MBs, ragged right/bottom edges, several SA sizes);
+BASELINE.json's full sizes compare sampled MBs (corners, edges, stripe rows,
+seeded random rows) in the same launch configuration bench.py times.
+"""
+import numpy as np
+import pytest
+import torch
+
+from synth import CONFIGS, gen_flat, gen_noise, gen_shifted, gen_tex, make_workload
+
+pytestmark = pytest.mark.gpu
+
+GEN = {"tex": gen_tex, "noise": gen_noise, "flat": gen_flat}
+
+
+@pytest.fixture(scope="module")
+def feves():
+    import __graft_entry__ as g
+    g.build()
+    import paper_conf_icpp_ilicmrs14_b200 as pkg
+    assert torch.cuda.is_available()
+    return pkg
+
+
+def _dev(a):
+    return torch.from_numpy(np.ascontiguousarray(a)).cuda()
+
+
+def _frames(kind, W, H, n_rf, seed):
+    g = GEN[kind]
+    cf = g(W, H, n_rf, seed)
+    rfs = [g(W, H, n_rf - 1 - k, seed) for k in range(n_rf)]
+    return cf, rfs
+
+
+def _run_me(feves, cf, rfs, S):
+    H, W = cf.shape
+    me = feves.MotionEstimator(W, H, S, len(rfs))
+    mvs, sads = me.estimate(_dev(cf), [_dev(r) for r in rfs])
+    torch.cuda.synchronize()
+    n = me.mb_rows * me.mb_cols
+    out = mvs.cpu().numpy().reshape(n, len(rfs), 41, 2), sads.cpu().numpy().reshape(n, len(rfs), 41)
+    me.close()
+    return out
+
+
+SMALL = [  # (W, H, S, n_rf, kind)
+    (64, 48, 16, 1, "tex"), (64, 48, 16, 2, "noise"), (80, 40, 8, 1, "flat"),
+    (72, 52, 32, 2, "tex"),            # ragged: 72 = 4.5 MBs, 52 = 3.25 MBs
+    (100, 36, 4, 3, "noise"), (50, 30, 6, 1, "tex"), (96, 80, 64, 1, "tex"),
+    (48, 48, 12, 2, "flat"), (40, 40, 128, 1, "noise"),
+]
+
+
+@pytest.mark.parametrize("W,H,S,n_rf,kind", SMALL)
+def test_me_full_frame_small(feves, orc, W, H, S, n_rf, kind):
+    cf, rfs = _frames(kind, W, H, n_rf, 1000 + W + S)
+    g_mvs, g_sads = _run_me(feves, cf, rfs, S)
+    o_mvs, o_sads = orc.me(cf, rfs, S)
+    np.testing.assert_array_equal(g_sads, o_sads)
+    np.testing.assert_array_equal(g_mvs, o_mvs)
+
+
+@pytest.mark.parametrize("kind", ["tex", "noise", "flat"])
+def test_me_cif_config(feves, orc, kind):
+    """BASELINE config 1: CIF 352x288, 2 frames, 1 RF, SA 16, full frame."""
+    cfg = CONFIGS["cif"]
+    cf, rfs = make_workload(cfg, kind=kind)
+    g_mvs, g_sads = _run_me(feves, cf, rfs, cfg.sa_range)
+    o_mvs, o_sads = orc.me(cf, rfs, cfg.sa_range)
+    np.testing.assert_array_equal(g_sads, o_sads)
+    np.testing.assert_array_equal(g_mvs, o_mvs)
+
+
+@pytest.mark.parametrize("uv", [(5, -3), (-8, 7)])
+def test_me_global_shift(feves, uv):
+    rf = gen_noise(128, 96, 0, 3)
+    cf = gen_shifted(rf, *uv)
+    g_mvs, g_sads = _run_me(feves, cf, [rf], 16)
+    interior = g_mvs.reshape(6, 8, 1, 41, 2)[1:-1, 1:-1]
+    assert (interior[..., 0] == uv[0]).all() and (interior[..., 1] == uv[1]).all()
+
+
+def test_me_identical_frames(feves):
+    f = gen_flat(96, 64, 0, 9)
+    g_mvs, g_sads = _run_me(feves, f, [f, f], 32)
+    assert (g_sads == 0).all() and (g_mvs == 0).all()
+
+
+@pytest.mark.parametrize("W,H,S", [(64, 48, 8), (72, 52, 16), (50, 30, 64), (33, 17, 128)])
+def test_int_planes_full(feves, orc, W, H, S):
+    rf = gen_noise(W, H, 0, W * H) if S != 16 else gen_tex(W, H, 0, 5)
+    me = feves.MotionEstimator(W, H, S, 1)
+    sf = me.interpolate(_dev(rf))
+    torch.cuda.synchronize()
+    pad, pitch, rows = orc.sf_layout(W, H, S)
+    assert (me.sf_pad, me.sf_pitch, me.sf_rows) == (pad, pitch, rows)
+    np.testing.assert_array_equal(sf.cpu().numpy(), orc.int_planes(rf, pad, pitch, rows))
+    me.close()
+
+
+@pytest.mark.parametrize("W,H,S,n_rf,kind", [(64, 48, 16, 2, "tex"), (72, 52, 8, 1, "noise"),
+                                             (80, 48, 32, 2, "flat"), (50, 30, 64, 1, "tex")])
+def test_sme_full_frame(feves, orc, W, H, S, n_rf, kind):
+    cf, rfs = _frames(kind, W, H, n_rf, 7 + S)
+    me = feves.MotionEstimator(W, H, S, n_rf)
+    tcf, trfs = _dev(cf), [_dev(r) for r in rfs]
+    sfs = [me.interpolate(r) for r in trfs]
+    mvs, sads = me.estimate(tcf, trfs)
+    q1, s1 = me.refine(tcf, sfs, mvs, sads)
+    q2, s2 = me.refine(tcf, sfs, mvs, None)          # centre recomputed from the SF
+    torch.cuda.synchronize()
+    n = me.mb_rows * me.mb_cols
+    o_mvs, _ = orc.me(cf, rfs, S)
+    o_q, o_s = orc.sme(cf, rfs, o_mvs)
+    np.testing.assert_array_equal(mvs.cpu().numpy().reshape(n, n_rf, 41, 2), o_mvs)
+    for q, s in ((q1, s1), (q2, s2)):
+        np.testing.assert_array_equal(s.cpu().numpy().reshape(n, n_rf, 41), o_s)
+        np.testing.assert_array_equal(q.cpu().numpy().reshape(n, n_rf, 41, 2), o_q)
+    me.close()
+
+
+def test_encode_frame_equals_separate_calls(feves):
+    W, H, S = 96, 64, 16
+    cf, rfs = _frames("tex", W, H, 2, 4)
+    me = feves.MotionEstimator(W, H, S, 2)
+    tcf, trfs = _dev(cf), [_dev(r) for r in rfs]
+    sfs_a = [me.interpolate(r) for r in trfs]
+    mvs, sads = me.estimate(tcf, trfs)
+    qa, sa = me.refine(tcf, sfs_a, mvs, sads)
+    sfs_b = [me.new_sf() for _ in trfs]
+    (m2, s2), (qb, sb) = me.encode_frame(tcf, trfs, sfs_b, n_int=2, out_me=me.new_mvs())
+    assert me.launches == 4
+    torch.cuda.synchronize()
+    assert torch.equal(mvs, m2) and torch.equal(sads, s2) and torch.equal(qa, qb) and torch.equal(sa, sb)
+    for a, b in zip(sfs_a, sfs_b):
+        assert torch.equal(a, b)
+    me.close()
+
+
+def test_host_pointer_rejected(feves):
+    me = feves.MotionEstimator(64, 48, 16, 1)
+    cf = torch.zeros(48, 64, dtype=torch.uint8)          # host tensor
+    with pytest.raises(feves.FevesError):
+        me.estimate(cf, [cf])
+    me.close()
+
+
+# ----------------------------------------------------- full BASELINE sizes --
+
+def _sample_mbs(mb_cols, mb_rows, n_random, seed, stripes=(2, 4, 8)):
+    rows = {0, mb_rows - 1}
+    for g in stripes:
+        base, extra = divmod(mb_rows, g)
+        r = 0
+        for i in range(g):
+            r += base + (1 if i < extra else 0)
+            rows |= {min(r, mb_rows - 1), max(r - 1, 0)}
+    rng = np.random.default_rng(seed)
+    mbs = {0, mb_cols - 1, (mb_rows - 1) * mb_cols, mb_rows * mb_cols - 1}
+    for r in rows:
+        mbs |= {r * mb_cols, r * mb_cols + mb_cols - 1, r * mb_cols + int(rng.integers(mb_cols))}
+    mbs |= set(int(v) for v in rng.integers(0, mb_rows * mb_cols, n_random))
+    return np.array(sorted(mbs), np.int32)
+
+
+@pytest.mark.parametrize("name,n_random", [("1080p_sa32", 24), ("1080p_sa64_4rf", 12), ("2160p_sa128", 3)])
+def test_full_size_sampled(feves, orc, name, n_random):
+    """Full BASELINE sizes through encode_frame (the launch bench.py times); sampled MBs."""
+    cfg = CONFIGS[name]
+    cf, rfs = make_workload(cfg, kind="tex")
+    me = feves.MotionEstimator(cfg.width, cfg.height, cfg.sa_range, cfg.n_rf)
+    tcf, trfs = _dev(cf), [_dev(r) for r in rfs]
+    sfs = [me.new_sf() for _ in trfs]
+    (mvs, sads), (qmvs, qsads) = me.encode_frame(tcf, trfs, sfs, n_int=cfg.n_rf, out_me=me.new_mvs())
+    torch.cuda.synchronize()
+    n = me.mb_rows * me.mb_cols
+    mvs = mvs.cpu().numpy().reshape(n, cfg.n_rf, 41, 2)
+    sads = sads.cpu().numpy().reshape(n, cfg.n_rf, 41)
+    qmvs = qmvs.cpu().numpy().reshape(n, cfg.n_rf, 41, 2)
+    qsads = qsads.cpu().numpy().reshape(n, cfg.n_rf, 41)
+    mbs = _sample_mbs(me.mb_cols, me.mb_rows, n_random, 5)
+    if name == "2160p_sa128":
+        mbs = mbs[np.random.default_rng(1).choice(len(mbs), 10, replace=False)]
+    o_mvs, o_sads = orc.me(cf, rfs, cfg.sa_range, mb_list=mbs)
+    np.testing.assert_array_equal(sads[mbs], o_sads)
+    np.testing.assert_array_equal(mvs[mbs], o_mvs)
+    o_q, o_qs = orc.sme(cf, rfs, o_mvs, mb_list=mbs)
+    np.testing.assert_array_equal(qsads[mbs], o_qs)
+    np.testing.assert_array_equal(qmvs[mbs], o_q)
+    # properties that hold everywhere
+    assert (qsads <= sads).all()
+    assert np.abs(qmvs.astype(np.int32) - 4 * mvs.astype(np.int32)).max() <= 3
+    # INT: sampled rows of the first SF (top margin, frame edge rows, bottom margin)
+    pad, pitch, rows = orc.sf_layout(cfg.width, cfg.height, cfg.sa_range)
+    sf0 = sfs[0].cpu().numpy()
+    for r in (0, pad - 1, pad, pad + cfg.height // 2, pad + cfg.height - 1, rows - 1):
+        ref = orc.int_planes(rfs[0], pad, pitch, rows, row_begin=r, row_end=r + 1)
+        np.testing.assert_array_equal(sf0[:, r], ref[:, r])
+    me.close()
+
+
+def test_determinism(feves):
+    cfg = CONFIGS["1080p_sa32"]
+    cf, rfs = make_workload(cfg, kind="flat")
+    a = _run_me(feves, cf, rfs, cfg.sa_range)
+    b = _run_me(feves, cf, rfs, cfg.sa_range)
+    np.testing.assert_array_equal(a[0], b[0])
+    np.testing.assert_array_equal(a[1], b[1])
+
+
+@pytest.mark.parametrize("g", [2, 3, 8])
+def test_stripes_virtual_ranks(feves, g):
+    """P11 on the GPU: me_set_rows stripes (as the ranks of a G-GPU run would) == full frame."""
+    W, H, S, n_rf = 320, 200, 32, 2     # 13 MB rows, ragged bottom
+    cf, rfs = _frames("tex", W, H, n_rf, 42)
+    me = feves.MotionEstimator(W, H, S, n_rf)
+    tcf, trfs = _dev(cf), [_dev(r) for r in rfs]
+    sfs = [me.new_sf() for _ in trfs]
+    (fm, fs), (fq, fqs) = me.encode_frame(tcf, trfs, sfs, n_int=n_rf, out_me=me.new_mvs())
+    base, extra = divmod(me.mb_rows, g)
+    r0 = 0
+    for i in range(g):
+        r1 = r0 + base + (1 if i < extra else 0)
+        me.set_rows(r0, r1)
+        sfs_s = [me.new_sf() for _ in trfs]
+        (m, s), (q, qs) = me.encode_frame(tcf, trfs, sfs_s, n_int=n_rf, out_me=me.new_mvs())
+        assert torch.equal(m, fm[r0:r1]) and torch.equal(s, fs[r0:r1])
+        assert torch.equal(q, fq[r0:r1]) and torch.equal(qs, fqs[r0:r1])
+        r0 = r1
+    me.close()
