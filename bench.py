@@ -1,0 +1,362 @@
+#!/usr/bin/env python
+"""bench.py -- FEVES inter-prediction hot path (ME + INT + SME) on B200.
+
+Metric (BASELINE.json): "1080p frames/s and candidate GSAD/s (ME+INT+SME) at
+1/2/4/8 B200".  One STEP = one IPPP inter-frame ("IPPP", P:323 one new
+RF per frame): INT of the newest RF || integer FSBM ME of the CF over its
+n_rf RFs (41 partitions) -> SME of all 41 x n_rf MVs, i.e. every row of
+SURVEY §8(a), through me_stream_push of libfeves_me.so.  Workload at N=1:
+BASELINE config[2] "1080p, 4 RFs, SA 64x64, ME + INT + SME, 1 B200"; at N>1
+config[3] (same frame, MB-row sharded, strong scaling).
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl feves|reference]
+
+Timing: W untimed warm-up steps after the RF ring is full; K timed steps,
+each bracketed by CUDA events on the context stream, L2 flushed (a 512 MiB
+write) before every timed step, barrier + synchronize around the region, max
+over ranks.  ``value`` = frames/s with inputs resident in HBM; ``e2e`` = the
+same through the C-ABI with pinned HOST buffers (H2D of the frame and D2H of
+the quarter-pel MVs + SADs inside every step).  ``--impl reference`` times
+the CPU oracle (oracle/) on a bounded MB sample of the same workload.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "1080p frames/s and candidate GSAD/s (ME+INT+SME) at 1/2/4/8 B200"
+N_SM = 148
+PX_PER_CLK_SM = 256          # 64 VABSDIFF4 lanes/clk/SM x 4 px (profiles/r01/int_peaks.json)
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=200)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", choices=["feves", "reference"], default="feves")
+    ap.add_argument("--config", default=None, help="synth.CONFIGS key (default: by --gpus)")
+    ap.add_argument("--e2e-steps", type=int, default=50)
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--cpu-budget", type=float, default=10.0, help="seconds of oracle wall time")
+    return ap.parse_args()
+
+
+def peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            return json.load(f), "measured"
+    except OSError:
+        return {"hbm_gbs": 6650.0, "sm_max_mhz": 1965.0}, "fallback"
+
+
+def workload_units(cfg, n_ref=None):
+    """Algorithmic work of one frame."""
+    mbc, mbr = -(-cfg.width // 16), -(-cfg.height // 16)
+    n_ref = cfg.n_rf if n_ref is None else n_ref
+    n_mb = mbc * mbr
+    me_cands = n_mb * n_ref * cfg.sa_range ** 2           # MB-candidates (each 256 px-absdiff, 41 SADs)
+    sme_px = n_mb * n_ref * 16 * 7 * 256                   # 16 sub-pel candidates x 7 modes x 256 px
+    R = cfg.sa_range // 2
+    pad = -(-(R + 4) // 16) * 16
+    sf_bytes = 16 * (16 * mbr + 2 * pad) * (16 * mbc + 2 * pad)
+    int_bytes = cfg.width * cfg.height + sf_bytes          # read the RF, write 16 planes
+    return dict(n_mb=n_mb, me_cands=me_cands, me_px=me_cands * 256, sme_px=sme_px,
+                gsad=me_cands + sme_px / 256, int_bytes=int_bytes)
+
+
+class Clocks:
+    """nvidia-smi sampler for the timed region (B200_PROFILING.md clocks line)."""
+
+    Q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index):
+        self.index = index
+        self.p = None
+
+    def start(self):
+        try:
+            self.p = subprocess.Popen(["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.Q}",
+                                       "--format=csv,noheader,nounits", "-lms", "50"],
+                                      stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            time.sleep(0.3)
+        except OSError:
+            self.p = None
+
+    def stop(self):
+        if self.p is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.p.terminate()
+        out, _ = self.p.communicate(timeout=10)
+        sm, mx, reasons = [], None, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for line in out.strip().splitlines():
+            f = [x.strip() for x in line.split(",")]
+            if len(f) < 7:
+                continue
+            try:
+                sm.append(float(f[0]))
+                mx = float(f[1])
+            except ValueError:
+                continue
+            for n, v in zip(names, f[3:7]):
+                if v.lower().startswith("active"):
+                    reasons.add(n)
+        busy = [s for s in sm if s > 300] or sm
+        return {"sm_mhz": statistics.median(busy) if busy else None, "sm_max_mhz": mx,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+# ----------------------------------------------------------------- reference --
+
+class OracleSampler:
+    """The oracle (as it stands, never tuned) on a bounded seeded MB sample of one frame."""
+
+    def __init__(self, cfg):
+        import numpy as np
+        import oracle
+        from synth import make_workload
+
+        oracle.build()
+        self.orc, self.cfg = oracle, cfg
+        self.threads = os.cpu_count() or 1
+        self.cf, self.rfs = make_workload(cfg)
+        self.n_total = workload_units(cfg)["n_mb"]
+        self.order = np.random.default_rng(1234).permutation(self.n_total).astype(np.int32)
+        self.layout = oracle.sf_layout(cfg.width, cfg.height, cfg.sa_range)
+        t0 = time.perf_counter()              # calibrate: one MB per thread
+        self.run(self.threads)
+        self.t_cal = time.perf_counter() - t0
+
+    def size_for(self, budget_s):
+        n = self.threads * max(1, round(budget_s / max(self.t_cal, 1e-3)))
+        return int(min(self.n_total, n))
+
+    def run(self, n):
+        import numpy as np
+        cfg, orc = self.cfg, self.orc
+        mbs = np.sort(self.order[:n])
+        pad, pitch, rows = self.layout
+        int_rows = max(1, round(rows * n / self.n_total))
+        t0 = time.perf_counter()
+        mv, _ = orc.me(self.cf, self.rfs, cfg.sa_range, mb_list=mbs, threads=self.threads)
+        t1 = time.perf_counter()
+        orc.sme(self.cf, self.rfs, mv, mb_list=mbs, threads=self.threads)
+        t2 = time.perf_counter()
+        orc.int_planes(self.rfs[0], pad, pitch, rows, row_begin=0, row_end=int_rows, threads=self.threads)
+        t3 = time.perf_counter()
+        t = t3 - t0
+        fps = (n / self.n_total) / t
+        return {"value": fps, "unit": "frames/s", "cores": self.threads, "kind": "oracle",
+                "sample": f"{n} of {self.n_total} MBs (seeded) x {cfg.n_rf} RFs ME+SME and {int_rows} of {rows} "
+                          f"SF rows of one INT ({t:.1f} s wall on {self.threads} threads), extrapolated linearly "
+                          f"(FSBM work is linear in MBs, P:260)",
+                "seconds": {"me": t1 - t0, "sme": t2 - t1, "int": t3 - t2},
+                "candidate_gsad_per_s": workload_units(cfg)["gsad"] * fps / 1e9}
+
+
+def cpu_oracle_sample(cfg, budget_s):
+    s = OracleSampler(cfg)
+    return s.run(s.size_for(budget_s))
+
+
+def run_reference(args, cfg):
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    s = OracleSampler(cfg)
+    n = s.size_for(min(args.cpu_budget, 150.0 / (args.steps + args.warmup)))
+    vals, cb = [], None
+    for i in range(args.warmup + args.steps):
+        cb = s.run(n)
+        if i >= args.warmup:
+            vals.append(cb["value"])
+    v = statistics.mean(vals)
+    line = {"impl": "reference", "metric": METRIC, "value": v, "unit": "frames/s", "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 / v, "higher_is_better": True,
+            "scaling": "strong" if args.gpus > 1 else "weak", "vs_baseline": None, "dtype": "u8",
+            "data": "synthetic (gen-tex, seeded)", "config": config_json(cfg, args),
+            "cpu_baseline": {"kind": cb["kind"], "cores": cb["cores"], "sample": cb["sample"], "value": v,
+                             "unit": "frames/s"},
+            "e2e": {"value": v, "unit": "frames/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+            "candidate_gsad_per_s": workload_units(cfg)["gsad"] * v / 1e9}
+    print(json.dumps(line), flush=True)
+
+
+def config_json(cfg, args):
+    return {"workload": cfg.name, "baseline_config_index": cfg.baseline_index, "width": cfg.width,
+            "height": cfg.height, "n_rf": cfg.n_rf, "sa_range": cfg.sa_range, "path": "int+me+sme (IPPP stream)",
+            "partitions": 41, "parallelism": f"mb-row x{args.gpus}", "l2": "flushed (512 MiB write) before every timed step"}
+
+
+# --------------------------------------------------------------------- feves --
+
+def run_feves(args, cfg):
+    import torch
+    import torch.distributed as dist
+
+    import __graft_entry__ as ge
+    ge.build()
+    import paper_conf_icpp_ilicmrs14_b200 as feves
+    from paper_conf_icpp_ilicmrs14_b200.shard import ShardedStream, stripes
+    from synth import ippp_sequence
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    me = feves.MotionEstimator(cfg.width, cfg.height, cfg.sa_range, cfg.n_rf, device=dev)
+    r0, r1 = stripes(me.mb_rows, world)[rank]
+    me.set_rows(r0, r1)
+    me.set_timing(True)
+    stream = torch.cuda.current_stream(dev)
+
+    n_frames = cfg.n_rf + 4
+    host = ippp_sequence(cfg.width, cfg.height, n_frames, 1000 + cfg.baseline_index)
+    frames = [torch.from_numpy(f).to(dev) for f in host]
+    pinned = [torch.from_numpy(f).pin_memory() for f in host]
+    buf = torch.empty_like(frames[0])
+    flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
+    ss = ShardedStream(me) if world > 1 else None
+
+    def push(t):
+        if ss is not None:
+            return ss.push(frames[t % n_frames], buf)
+        return me.stream_push(frames[t % n_frames], out=out_dev)
+
+    out_dev = me.new_mvs()
+    me.stream_reset()
+    t = 0
+    while t < cfg.n_rf + args.warmup:        # fill the RF/SF ring (P:323 ramp), then warm up
+        push(t)
+        t += 1
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    mod = []
+    clocks = Clocks(local)
+    clocks.start()
+    for k in range(args.steps):
+        flush.fill_(k & 0xff)
+        ev[k][0].record(stream)
+        push(t)
+        ev[k][1].record(stream)
+        t += 1
+        mod.append(me.timings())             # waits for this step's module events
+    torch.cuda.synchronize()
+    ck = clocks.stop()
+    step_ms = [a.elapsed_time(b) for a, b in ev]
+    tot = torch.tensor([sum(step_ms)], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(tot, op=dist.ReduceOp.MAX)
+        dist.barrier()
+    total_ms = float(tot.item())
+    fps = args.steps / (total_ms / 1e3)
+
+    u = workload_units(cfg)
+    int_ms = statistics.mean(m[0] for m in mod)
+    me_ms = statistics.mean(m[1] for m in mod)
+    sme_ms = statistics.mean(m[2] for m in mod)
+    stripe_frac = (r1 - r0) / me.mb_rows
+    pk, pk_src = peaks()
+    peak_px = N_SM * PX_PER_CLK_SM * pk.get("sm_max_mhz", 1965.0) * 1e6
+    achieved_px = u["me_px"] * stripe_frac / (me_ms / 1e3)
+    traffic = None
+    try:
+        with open(os.path.join(ROOT, "profiles", "ncu_traffic.json")) as f:
+            tr = json.load(f).get(cfg.name, {})
+            traffic = tr.get("me_fsbm_dram_bytes_per_launch")
+    except OSError:
+        pass
+
+    # ---- e2e: pinned host frame in, host MVs/SADs out, every step ----
+    e2e = None
+    if not args.no_e2e and world == 1:
+        qm_h = torch.empty(me.mv_shape() + (2,), dtype=torch.int16).pin_memory()
+        qs_h = torch.empty(me.mv_shape(), dtype=torch.uint16).pin_memory()
+        me.stream_reset()
+        for i in range(cfg.n_rf + 2):
+            me.stream_push(pinned[i % n_frames], out=(qm_h, qs_h))
+        me.sync()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        for i in range(args.e2e_steps):
+            me.stream_push(pinned[(cfg.n_rf + 2 + i) % n_frames], out=(qm_h, qs_h))
+        e1.record(stream)
+        me.sync()
+        torch.cuda.synchronize()
+        e2e_ms = e0.elapsed_time(e1)
+        e2e = {"value": args.e2e_steps / (e2e_ms / 1e3), "unit": "frames/s",
+               "h2d_bytes_per_step": pinned[0].numel(),
+               "d2h_bytes_per_step": qm_h.numel() * 2 + qs_h.numel() * 2,
+               "api": "me_stream_push(cf_on_host=1, out_on_host=1), pinned buffers, C-ABI"}
+
+    if rank != 0:
+        if world > 1:
+            dist.destroy_process_group()
+        return
+    cpu = None
+    if not args.no_cpu_baseline and world == 1:
+        cpu = cpu_oracle_sample(cfg, args.cpu_budget)
+    line = {
+        "metric": METRIC, "value": fps, "unit": "frames/s", "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": total_ms / args.steps, "higher_is_better": True,
+        "scaling": "strong" if world > 1 else "weak", "vs_baseline": None, "dtype": "u8",
+        "data": "synthetic (gen-tex: 8 sinusoids in (1.25,-0.75) px/frame motion + noise, seeded)",
+        "config": config_json(cfg, args),
+        "candidate_gsad_per_s": u["gsad"] * fps / 1e9,
+        "px_absdiff_per_s": (u["me_px"] + u["sme_px"]) * fps,
+        "kernels_ms": {"int": int_ms, "me": me_ms, "sme": sme_ms,
+                       "note": "CUDA events around each launch on its own stream (INT runs concurrently with ME)"},
+        "clocks": ck,
+        "e2e": e2e,
+        "gpu_launches": 3 * args.steps,
+        "roofline": {"bound": "alu", "kernel": "me_fsbm_kernel", "achieved": achieved_px / 1e12,
+                     "peak": peak_px / 1e12, "unit": "Tpx-absdiff/s", "frac": achieved_px / peak_px,
+                     "traffic": traffic,
+                     "peak_source": f"148 SM x 64 VABSDIFF4 lanes/clk x 4 px x sm_max_mhz ({pk_src} "
+                                    "MEASURED_PEAKS.json); issue rate measured in profiles/r01/int_peaks.json",
+                     "frac_at_observed_clock": (achieved_px / (N_SM * PX_PER_CLK_SM * ck["sm_mhz"] * 1e6))
+                     if ck.get("sm_mhz") else None},
+        "roofline_int": {"bound": "hbm", "kernel": "int_subpel_kernel",
+                         "achieved": u["int_bytes"] * stripe_frac / (int_ms / 1e3) / 1e9,
+                         "peak": pk.get("hbm_gbs", 6650.0), "unit": "GB/s",
+                         "frac": u["int_bytes"] * stripe_frac / (int_ms / 1e3) / 1e9 / pk.get("hbm_gbs", 6650.0)},
+        "cpu_baseline": cpu,
+    }
+    print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
+def main():
+    args = parse()
+    from synth import CONFIGS
+    name = args.config or ("1080p_sa64_4rf" if args.gpus == 1 else "1080p_shard")
+    cfg = CONFIGS[name]
+    if args.warmup < 3:
+        raise SystemExit("--warmup must be >= 3")
+    if args.impl == "reference":
+        run_reference(args, cfg)
+    else:
+        run_feves(args, cfg)
+
+
+if __name__ == "__main__":
+    main()

@@ -52,8 +52,15 @@ def lib():
         L.sme_refine.argtypes = [P, P, P, P, P, P, P]
         L.me_encode_frame.argtypes = [P, P, P, P, i, P, P, P, P]
         L.me_last_launch_count.argtypes = [P]
+        L.me_stream_reset.argtypes = [P]
+        L.me_stream_push.argtypes = [P, P, i, P, P, i, P]
+        L.me_stream_outputs.argtypes = [P, P, P]
+        L.me_sync.argtypes = [P]
+        L.me_set_timing.argtypes = [P, i]
+        L.me_get_timings.argtypes = [P, P, P, P]
         for fn in ("me_set_stream", "me_set_rows", "me_get_layout", "me_estimate", "int_interpolate",
-                   "sme_refine", "me_encode_frame", "me_last_launch_count"):
+                   "sme_refine", "me_encode_frame", "me_last_launch_count", "me_stream_reset",
+                   "me_stream_push", "me_stream_outputs", "me_sync", "me_set_timing", "me_get_timings"):
             getattr(L, fn).restype = i
         _lib = L
     return _lib
@@ -174,6 +181,39 @@ class MotionEstimator:
                                      None if sads is None else sads.data_ptr(),
                                      qmvs.data_ptr(), qsads.data_ptr()))
         return (mvs, sads), (qmvs, qsads)
+
+    # ------------------------------------------------------- IPPP stream --
+    def stream_reset(self):
+        _check(lib().me_stream_reset(self._ctx))
+
+    def stream_push(self, cf, out=None, bind_stream=True):
+        """Push frame t (device or pinned host uint8 tensor [H, W]) through
+        INT(t-1) || ME(t) -> SME(t) (me_stream_push).  Returns (qmvs, qsads,
+        n_ref_used); outputs live where ``out`` lives (device or host)."""
+        if not (isinstance(cf, torch.Tensor) and cf.dtype == torch.uint8 and cf.is_contiguous()):
+            raise FevesError("cf: expected a contiguous uint8 tensor")
+        on_host = not cf.is_cuda
+        qmvs, qsads = out if out is not None else self.new_mvs()
+        out_host = not qmvs.is_cuda
+        n = ctypes.c_int()
+        if bind_stream:
+            self._bind_stream()
+        _check(lib().me_stream_push(self._ctx, cf.data_ptr(), int(on_host), qmvs.data_ptr(), qsads.data_ptr(),
+                                    int(out_host), ctypes.byref(n)))
+        return qmvs, qsads, n.value
+
+    def sync(self):
+        _check(lib().me_sync(self._ctx))
+
+    # ---------------------------------------------- module timers (P:87) --
+    def set_timing(self, on: bool = True):
+        _check(lib().me_set_timing(self._ctx, int(on)))
+
+    def timings(self):
+        """(ms_int, ms_me, ms_sme) of the last call; -1 for modules it did not run."""
+        v = [ctypes.c_float() for _ in range(3)]
+        _check(lib().me_get_timings(self._ctx, *[ctypes.byref(x) for x in v]))
+        return tuple(x.value for x in v)
 
 
 __all__ = ["MotionEstimator", "FevesError", "lib", "LIB_PATH", "N_PART", "N_PHASE"]

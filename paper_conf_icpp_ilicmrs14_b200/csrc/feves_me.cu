@@ -35,9 +35,22 @@ struct me_ctx {
   int last_launches;
   const void* checked[64];
   int n_checked;
+  // IPPP stream state (me_stream_push): ring of n_rf+1 frames, n_rf SFs
+  uint8_t* ring;         // (n_rf+1) * W*H
+  uint8_t* sf_ring;      // n_rf * 16*sf_rows*sf_pitch
+  int16_t* d_qmvs;       // device outputs of the last push
+  uint16_t* d_qsads;
+  long long t;           // frames pushed since reset
+  cudaStream_t side;     // INT runs here, concurrently with ME
+  cudaEvent_t ev_fork, ev_join;
+  // per-module timers ("facilities to measure execution ... times")
+  int timing;
+  cudaEvent_t ev_t[6];   // INT start/stop (side stream), ME start/stop, SME start/stop
+  int timed_mask;        // which pairs were recorded by the last push/encode
 };
 
 static thread_local int g_last_error = ME_OK;
+constexpr int kNPhase = 16;
 
 // ------------------------------------------------------------- helpers ----
 static int spiral_rank_closed_form(int dx, int dy) {   // G4
@@ -134,6 +147,15 @@ extern "C" void me_destroy(me_ctx* c) {
   cudaFree(c->d_inv);
   cudaFree(c->d_mvs);
   cudaFree(c->d_sads);
+  cudaFree(c->ring);
+  cudaFree(c->sf_ring);
+  cudaFree(c->d_qmvs);
+  cudaFree(c->d_qsads);
+  for (int i = 0; i < 6; ++i)
+    if (c->ev_t[i]) cudaEventDestroy(c->ev_t[i]);
+  if (c->side) cudaStreamDestroy(c->side);
+  if (c->ev_fork) cudaEventDestroy(c->ev_fork);
+  if (c->ev_join) cudaEventDestroy(c->ev_join);
   if (c->own_stream && c->stream) cudaStreamDestroy(c->stream);
   delete c;
 }
@@ -179,24 +201,31 @@ extern "C" int me_get_layout(const me_ctx* c, int* mb_cols, int* mb_rows, int* s
 extern "C" int me_last_launch_count(const me_ctx* c) { return c ? c->last_launches : -1; }
 
 // --------------------------------------------------------------- launches ----
-static int launch_me(me_ctx* c, const uint8_t* cf, const uint8_t* const* rfs, int16_t* mvs, uint16_t* sads) {
+static void tmark(me_ctx* c, int i, cudaStream_t st) {
+  if (c->timing) { cudaEventRecord(c->ev_t[i], st); c->timed_mask |= 1 << (i / 2); }
+}
+
+static int launch_me(me_ctx* c, const uint8_t* cf, const uint8_t* const* rfs, int16_t* mvs, uint16_t* sads,
+                     int n_ref, cudaStream_t st) {
   MeParams P;
   memset(&P, 0, sizeof(P));
   P.cf = cf;
-  for (int k = 0; k < c->n_rf; ++k) P.rf[k] = rfs[k];
-  P.W = c->W; P.H = c->H; P.S = c->S; P.R = c->R; P.n_rf = c->n_rf;
+  for (int k = 0; k < n_ref; ++k) P.rf[k] = rfs[k];
+  P.W = c->W; P.H = c->H; P.S = c->S; P.R = c->R; P.n_rf = n_ref; P.rf_stride = c->n_rf;
   P.mb_cols = c->mb_cols; P.row0 = c->row0;
   P.rank_tab = c->d_rank; P.inv_tab = c->d_inv;
   P.out_mvs = mvs; P.out_sads = sads;
   P.lx = c->lx; P.ngx = c->ngx; P.nsub = c->nsub; P.nwy = c->nwy; P.dyl = c->dyl;
   P.pw = c->pw; P.cstride = c->cstride;
   dim3 grid(c->mb_cols, c->row1 - c->row0);
-  me_fsbm_kernel<<<grid, c->me_threads, c->me_smem, c->stream>>>(P);
+  tmark(c, 2, st);
+  me_fsbm_kernel<<<grid, c->me_threads, c->me_smem, st>>>(P);
+  tmark(c, 3, st);
   c->last_launches++;
   return launch_status();
 }
 
-static int launch_int(me_ctx* c, const uint8_t* rf, uint8_t* sf) {
+static int launch_int(me_ctx* c, const uint8_t* rf, uint8_t* sf, cudaStream_t st) {
   IntParams P;
   P.rf = rf; P.sf = sf; P.W = c->W; P.H = c->H;
   P.pad = c->sf_pad; P.pitch = c->sf_pitch; P.rows = c->sf_rows;
@@ -210,27 +239,31 @@ static int launch_int(me_ctx* c, const uint8_t* rf, uint8_t* sf) {
   const int groups = c->sf_pitch / 16;
   dim3 block(32, 4);
   dim3 grid((groups + 31) / 32, (P.row_end - P.row_begin + 3) / 4);
-  int_subpel_kernel<<<grid, block, 0, c->stream>>>(P);
+  tmark(c, 0, st);
+  int_subpel_kernel<<<grid, block, 0, st>>>(P);
+  tmark(c, 1, st);
   c->last_launches++;
   return launch_status();
 }
 
 static int launch_sme(me_ctx* c, const uint8_t* cf, const uint8_t* const* sfs, const int16_t* in_mvs,
-                      const uint16_t* in_sads, int16_t* out_qmvs, uint16_t* out_sads) {
+                      const uint16_t* in_sads, int16_t* out_qmvs, uint16_t* out_sads, int n_ref, cudaStream_t st) {
   SmeParams P;
   memset(&P, 0, sizeof(P));
   P.cf = cf;
-  for (int k = 0; k < c->n_rf; ++k) P.sf[k] = sfs[k];
+  for (int k = 0; k < n_ref; ++k) P.sf[k] = sfs[k];
   P.in_mvs = reinterpret_cast<const uint32_t*>(in_mvs);
   P.in_sads = in_sads;
   P.out_qmvs = reinterpret_cast<uint32_t*>(out_qmvs);
   P.out_sads = out_sads;
-  P.W = c->W; P.H = c->H; P.n_rf = c->n_rf; P.mb_cols = c->mb_cols; P.row0 = c->row0;
-  P.n_items = (c->row1 - c->row0) * c->mb_cols * c->n_rf;
+  P.W = c->W; P.H = c->H; P.n_rf = n_ref; P.rf_stride = c->n_rf; P.mb_cols = c->mb_cols; P.row0 = c->row0;
+  P.n_items = (c->row1 - c->row0) * c->mb_cols * n_ref;
   P.pad = c->sf_pad; P.pitch = c->sf_pitch;
   P.plane = (size_t)c->sf_rows * c->sf_pitch;
   const int per_block = 128 / 16;
-  sme_refine_kernel<<<(P.n_items + per_block - 1) / per_block, 128, 0, c->stream>>>(P);
+  tmark(c, 4, st);
+  sme_refine_kernel<<<(P.n_items + per_block - 1) / per_block, 128, 0, st>>>(P);
+  tmark(c, 5, st);
   c->last_launches++;
   return launch_status();
 }
@@ -243,13 +276,13 @@ extern "C" int me_estimate(me_ctx* c, const uint8_t* cf, const uint8_t* const* r
   for (int k = 0; k < c->n_rf; ++k)
     if (!is_device_ptr(c, rfs[k])) return ME_EINVAL;
   c->last_launches = 0;
-  return launch_me(c, cf, rfs, out_mvs, out_sads);
+  return launch_me(c, cf, rfs, out_mvs, out_sads, c->n_rf, c->stream);
 }
 
 extern "C" int int_interpolate(me_ctx* c, const uint8_t* rf, uint8_t* out_sf) {
   if (!c || !is_device_ptr(c, rf) || !is_device_ptr(c, out_sf)) return ME_EINVAL;
   c->last_launches = 0;
-  return launch_int(c, rf, out_sf);
+  return launch_int(c, rf, out_sf, c->stream);
 }
 
 extern "C" int sme_refine(me_ctx* c, const uint8_t* cf, const uint8_t* const* sfs, const int16_t* in_mvs,
@@ -262,7 +295,7 @@ extern "C" int sme_refine(me_ctx* c, const uint8_t* cf, const uint8_t* const* sf
   for (int k = 0; k < c->n_rf; ++k)
     if (!is_device_ptr(c, sfs[k])) return ME_EINVAL;
   c->last_launches = 0;
-  return launch_sme(c, cf, sfs, in_mvs, in_sads, out_qmvs, out_sads);
+  return launch_sme(c, cf, sfs, in_mvs, in_sads, out_qmvs, out_sads, c->n_rf, c->stream);
 }
 
 extern "C" int me_encode_frame(me_ctx* c, const uint8_t* cf, const uint8_t* const* rfs, uint8_t* const* sfs,
@@ -276,9 +309,126 @@ extern "C" int me_encode_frame(me_ctx* c, const uint8_t* cf, const uint8_t* cons
   int16_t* mvs = out_mvs ? out_mvs : c->d_mvs;
   uint16_t* sads = out_sads ? out_sads : c->d_sads;
   c->last_launches = 0;
+  c->timed_mask = 0;
   int st;
   for (int k = 0; k < n_int; ++k)
-    if ((st = launch_int(c, rfs[k], sfs[k])) != ME_OK) return st;
-  if ((st = launch_me(c, cf, rfs, mvs, sads)) != ME_OK) return st;
-  return launch_sme(c, cf, reinterpret_cast<const uint8_t* const*>(sfs), mvs, sads, out_qmvs, out_qsads);
+    if ((st = launch_int(c, rfs[k], sfs[k], c->stream)) != ME_OK) return st;
+  if ((st = launch_me(c, cf, rfs, mvs, sads, c->n_rf, c->stream)) != ME_OK) return st;
+  return launch_sme(c, cf, reinterpret_cast<const uint8_t* const*>(sfs), mvs, sads, out_qmvs, out_qsads, c->n_rf,
+                    c->stream);
+}
+
+// ------------------------------------------------------------ IPPP stream ----
+// frames are encoded in order (frame t needs the RFs reconstructed from
+// t-1, t-2, ...); the number of usable RFs ramps up over the first
+// frames; "ME and INT can be simultaneously processed".  Here the RF of
+// frame t-1 is the frame itself (no R* reconstruction on this path, DESIGN.md
+// §9).  Push of frame t: copy it into ring slot t mod (n_rf+1); INT(frame t-1)
+// into SF slot (t-1) mod n_rf on the side stream, concurrently with ME of frame
+// t over its min(t, n_rf) RFs; join; SME; outputs (quarter-pel MVs + SADs).
+extern "C" int me_stream_reset(me_ctx* c) {
+  if (!c) return ME_EINVAL;
+  c->t = 0;
+  return ME_OK;
+}
+
+static int stream_alloc(me_ctx* c) {
+  if (c->ring) return ME_OK;
+  const size_t fb = (size_t)c->W * c->H, sb = (size_t)kNPhase * c->sf_rows * c->sf_pitch;
+  const size_t nmv = (size_t)c->mb_cols * c->mb_rows * c->n_rf * kNPart;
+  if (cudaMalloc(&c->ring, fb * (c->n_rf + 1)) != cudaSuccess ||
+      cudaMalloc(&c->sf_ring, sb * c->n_rf) != cudaSuccess || cudaMalloc(&c->d_qmvs, nmv * 4) != cudaSuccess ||
+      cudaMalloc(&c->d_qsads, nmv * 2) != cudaSuccess ||
+      cudaStreamCreateWithFlags(&c->side, cudaStreamNonBlocking) != cudaSuccess ||
+      cudaEventCreateWithFlags(&c->ev_fork, cudaEventDisableTiming) != cudaSuccess ||
+      cudaEventCreateWithFlags(&c->ev_join, cudaEventDisableTiming) != cudaSuccess) {
+    cudaGetLastError();
+    return ME_ENOMEM;
+  }
+  return ME_OK;
+}
+
+extern "C" int me_stream_push(me_ctx* c, const uint8_t* cf, int cf_on_host, int16_t* out_qmvs,
+                              uint16_t* out_qsads, int out_on_host, int* n_ref_used) {
+  if (!c || !cf) return ME_EINVAL;
+  if (!cf_on_host && !is_device_ptr(c, cf)) return ME_EINVAL;
+  if (out_qmvs && !out_on_host && !is_device_ptr(c, out_qmvs)) return ME_EINVAL;
+  if (out_qsads && !out_on_host && !is_device_ptr(c, out_qsads)) return ME_EINVAL;
+  int st = stream_alloc(c);
+  if (st != ME_OK) return st;
+  c->last_launches = 0;
+  c->timed_mask = 0;
+  const size_t fb = (size_t)c->W * c->H, sb = (size_t)kNPhase * c->sf_rows * c->sf_pitch;
+  const int slots = c->n_rf + 1;
+  const long long t = c->t;
+  uint8_t* cur = c->ring + (size_t)(t % slots) * fb;
+  if (cudaMemcpyAsync(cur, cf, fb, cf_on_host ? cudaMemcpyHostToDevice : cudaMemcpyDeviceToDevice, c->stream) !=
+      cudaSuccess)
+    return launch_status();
+  const int n_ref = (int)std::min<long long>(t, c->n_rf);
+  if (n_ref_used) *n_ref_used = n_ref;
+  if (n_ref > 0) {
+    // side stream: INT of the newest RF (frame t-1), concurrent with ME
+    uint8_t* new_rf = c->ring + (size_t)((t - 1) % slots) * fb;
+    uint8_t* new_sf = c->sf_ring + (size_t)((t - 1) % c->n_rf) * sb;
+    if (cudaEventRecord(c->ev_fork, c->stream) != cudaSuccess ||
+        cudaStreamWaitEvent(c->side, c->ev_fork, 0) != cudaSuccess)
+      return launch_status();
+    if ((st = launch_int(c, new_rf, new_sf, c->side)) != ME_OK) return st;
+    if (cudaEventRecord(c->ev_join, c->side) != cudaSuccess) return launch_status();
+    const uint8_t* rfs[kMaxRf];
+    const uint8_t* sfs[kMaxRf];
+    for (int k = 0; k < n_ref; ++k) {           // ref_idx k = frame t-1-k
+      rfs[k] = c->ring + (size_t)((t - 1 - k) % slots) * fb;
+      sfs[k] = c->sf_ring + (size_t)((t - 1 - k) % c->n_rf) * sb;
+    }
+    if ((st = launch_me(c, cur, rfs, c->d_mvs, c->d_sads, n_ref, c->stream)) != ME_OK) return st;
+    if (cudaStreamWaitEvent(c->stream, c->ev_join, 0) != cudaSuccess) return launch_status();
+    int16_t* qm = (out_qmvs && !out_on_host) ? out_qmvs : c->d_qmvs;
+    uint16_t* qs = (out_qsads && !out_on_host) ? out_qsads : c->d_qsads;
+    if ((st = launch_sme(c, cur, sfs, c->d_mvs, c->d_sads, qm, qs, n_ref, c->stream)) != ME_OK) return st;
+    const size_t nmv = (size_t)(c->row1 - c->row0) * c->mb_cols * c->n_rf * kNPart;
+    if (out_on_host) {
+      if ((out_qmvs && cudaMemcpyAsync(out_qmvs, qm, nmv * 4, cudaMemcpyDeviceToHost, c->stream) != cudaSuccess) ||
+          (out_qsads && cudaMemcpyAsync(out_qsads, qs, nmv * 2, cudaMemcpyDeviceToHost, c->stream) != cudaSuccess))
+        return launch_status();
+    }
+  }
+  c->t = t + 1;
+  return ME_OK;
+}
+
+extern "C" int me_sync(me_ctx* c) {
+  if (!c) return ME_EINVAL;
+  return cudaStreamSynchronize(c->stream) == cudaSuccess ? ME_OK : ME_ECUDA;
+}
+
+extern "C" int me_stream_outputs(me_ctx* c, int16_t** qmvs, uint16_t** qsads) {
+  if (!c) return ME_EINVAL;
+  if (qmvs) *qmvs = c->d_qmvs;
+  if (qsads) *qsads = c->d_qsads;
+  return ME_OK;
+}
+
+extern "C" int me_set_timing(me_ctx* c, int on) {
+  if (!c) return ME_EINVAL;
+  if (on && !c->ev_t[0])
+    for (int i = 0; i < 6; ++i)
+      if (cudaEventCreate(&c->ev_t[i]) != cudaSuccess) { cudaGetLastError(); return ME_ENOMEM; }
+  c->timing = on ? 1 : 0;
+  return ME_OK;
+}
+
+extern "C" int me_get_timings(me_ctx* c, float* ms_int, float* ms_me, float* ms_sme) {
+  if (!c || !c->ev_t[0]) return ME_EINVAL;
+  float* out[3] = {ms_int, ms_me, ms_sme};
+  for (int k = 0; k < 3; ++k) {
+    if (!out[k]) continue;
+    *out[k] = -1.f;
+    if (!(c->timed_mask & (1 << k))) continue;
+    if (cudaEventSynchronize(c->ev_t[2 * k + 1]) != cudaSuccess ||
+        cudaEventElapsedTime(out[k], c->ev_t[2 * k], c->ev_t[2 * k + 1]) != cudaSuccess)
+      return launch_status();
+  }
+  return ME_OK;
 }

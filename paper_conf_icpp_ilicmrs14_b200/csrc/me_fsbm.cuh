@@ -34,7 +34,8 @@ constexpr int kMeT = 4;   // candidates per vertical step
 struct MeParams {
   const uint8_t* cf;
   const uint8_t* rf[kMaxRf];
-  int W, H, S, R, n_rf;
+  int W, H, S, R, n_rf;       // n_rf = RFs searched by this launch (RF ramp)
+  int rf_stride;              // RF dimension of the output layout (the context's n_rf)
   int mb_cols, row0;
   const uint32_t* rank_tab;   // [S][S], [dy+R][dx+R] -> spiral rank (G4)
   const uint32_t* inv_tab;    // rank -> (dx & 0xffff) | (dy << 16)
@@ -114,7 +115,6 @@ template <int BY>
 __device__ __forceinline__ void fold_pair(uint32_t (&M)[kNPart], const uint32_t (&Ka)[16], const uint32_t (&Kb)[16]) {
 #pragma unroll
   for (int s = 0; s < 16; ++s) {
-    constexpr int dummy = 0; (void)dummy;
     const int p = part_of(BY, s);
     if (p >= 0) M[p] = umin3(M[p], Ka[s], Kb[s]);
   }
@@ -219,7 +219,7 @@ __global__ void __launch_bounds__(256) me_fsbm_kernel(const MeParams P) {
       uint32_t k = red[p];
       for (int w = 1; w < nwarps; ++w) k = min(k, red[w * kNPart + p]);
       const uint32_t mv = __ldg(P.inv_tab + (k & 0xffffu));
-      const size_t o = ((size_t)(blockIdx.y * P.mb_cols + mbx) * P.n_rf + ref) * kNPart + p;
+      const size_t o = ((size_t)(blockIdx.y * P.mb_cols + mbx) * P.rf_stride + ref) * kNPart + p;
       reinterpret_cast<uint32_t*>(P.out_mvs)[o] = mv;
       P.out_sads[o] = (uint16_t)(k >> 16);
     }

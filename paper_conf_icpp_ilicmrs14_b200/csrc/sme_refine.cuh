@@ -25,7 +25,7 @@ struct SmeParams {
   const uint16_t* in_sads;    // may be null
   uint32_t* out_qmvs;
   uint16_t* out_sads;
-  int W, H, n_rf, mb_cols, row0, n_items;
+  int W, H, n_rf, rf_stride, mb_cols, row0, n_items;   // n_rf RFs refined, rf_stride = layout
   int pad, pitch;
   size_t plane;
 };
@@ -104,7 +104,7 @@ __global__ void __launch_bounds__(128) sme_refine_kernel(const SmeParams P) {
 #pragma unroll
   for (int r = 0; r < 4; ++r) cfb[r] = load4_clamped(P.cf, P.W, P.H, bxp, byp + r);
   const uint8_t* __restrict__ sf = P.sf[ref];
-  const size_t o = (size_t)item * kNPart;    // [mb][ref][41] with item = mb * n_rf + ref
+  const size_t o = ((size_t)mbi * P.rf_stride + ref) * kNPart;    // [mb][ref][41]
   const int s = 2 * by1 + bx1;
   refine_mode<15>(P, sf, 0, o, bxp, byp, b, cfb);                           // 16x16
   refine_mode<7>(P, sf, 1 + by1, o, bxp, byp, b, cfb);                      // 16x8

@@ -233,3 +233,46 @@ def test_stripes_virtual_ranks(feves, g):
         assert torch.equal(q, fq[r0:r1]) and torch.equal(qs, fqs[r0:r1])
         r0 = r1
     me.close()
+
+
+def test_stream_push_ippp(feves, orc):
+    """IPPP stream: frame t is searched over frames t-1..t-min(t,n_rf) (RF ramp)."""
+    W, H, S, n_rf = 80, 48, 16, 3
+    frames = [gen_tex(W, H, t, 61) for t in range(6)]
+    me = feves.MotionEstimator(W, H, S, n_rf)
+    n = me.mb_rows * me.mb_cols
+    for t, f in enumerate(frames):
+        qm, qs = me.new_mvs()
+        qm.fill_(-1)
+        qm, qs, used = me.stream_push(_dev(f), out=(qm, qs))
+        torch.cuda.synchronize()
+        assert used == min(t, n_rf)
+        if used == 0:
+            continue
+        rfs = [frames[t - 1 - k] for k in range(used)]
+        o_mvs, _ = orc.me(f, rfs, S)
+        o_q, o_s = orc.sme(f, rfs, o_mvs)
+        gq = qm.cpu().numpy().reshape(n, n_rf, 41, 2)
+        gs = qs.cpu().numpy().reshape(n, n_rf, 41)
+        np.testing.assert_array_equal(gq[:, :used], o_q)
+        np.testing.assert_array_equal(gs[:, :used], o_s)
+        assert (gq[:, used:] == -1).all()            # untouched
+    me.close()
+
+
+def test_stream_push_host_buffers(feves, orc):
+    W, H, S, n_rf = 64, 48, 8, 2
+    frames = [gen_noise(W, H, t, 3) for t in range(4)]
+    me = feves.MotionEstimator(W, H, S, n_rf)
+    n = me.mb_rows * me.mb_cols
+    out = (torch.empty(me.mv_shape() + (2,), dtype=torch.int16).pin_memory(),
+           torch.empty(me.mv_shape(), dtype=torch.uint16).pin_memory())
+    for t, f in enumerate(frames):
+        qm, qs, used = me.stream_push(torch.from_numpy(f).pin_memory(), out=out)
+        me.sync()
+    rfs = [frames[2], frames[1]]
+    o_mvs, _ = orc.me(frames[3], rfs, S)
+    o_q, o_s = orc.sme(frames[3], rfs, o_mvs)
+    np.testing.assert_array_equal(qm.numpy().reshape(n, n_rf, 41, 2), o_q)
+    np.testing.assert_array_equal(qs.numpy().reshape(n, n_rf, 41), o_s)
+    me.close()
