@@ -30,7 +30,7 @@ struct me_ctx {
   int16_t* d_mvs;        // scratch for me_encode_frame (full frame)
   uint16_t* d_sads;
   // ME launch geometry
-  int lx, ngx, nsub, nwy, dyl, pw, cstride, me_threads;
+  int me_threads;
   size_t me_smem;
   int last_launches;
   const void* checked[64];
@@ -73,6 +73,13 @@ static bool is_device_ptr(me_ctx* c, const void* p) {
   return true;
 }
 
+static cudaError_t set_me_smem(int bytes) {
+  cudaError_t e = cudaSuccess;
+  for (auto fn : {me_fsbm_kernel<0>, me_fsbm_kernel<16>, me_fsbm_kernel<32>, me_fsbm_kernel<64>, me_fsbm_kernel<128>})
+    if (e == cudaSuccess) e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
+  return e;
+}
+
 static int launch_status() {
   const cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) { fprintf(stderr, "feves_me: %s\n", cudaGetErrorString(e)); return ME_ECUDA; }
@@ -98,17 +105,8 @@ extern "C" me_ctx* me_create(int width, int height, int sa_range, int n_rf) {
   // lane geometry (me_fsbm.cuh): 32 dx per warp (fewer lanes per dx group for
   // small SAs, the rest of the warp takes other dy sub-ranges)
   const int S = c->S;
-  c->lx = S >= 32 ? 32 : S >= 16 ? 16 : S >= 8 ? 8 : 4;
-  c->ngx = (S + c->lx - 1) / c->lx;
-  c->nsub = 32 / c->lx;
-  c->nwy = 1;
-  const int parts = c->nsub * c->nwy;
-  c->dyl = ((S + parts - 1) / parts + kMeT - 1) / kMeT * kMeT;
-  c->pw = ((S - 1) >> 2) + 4;
-  const int words = (S + 15) * c->pw;
-  c->cstride = words + ((8 - words % 32) % 32 + 32) % 32;       // cstride = 8 (mod 32): conflict-free copies
-  c->me_threads = 32 * c->ngx * c->nwy;
-  c->me_smem = (size_t)(4 * c->cstride + (c->me_threads / 32) * kNPart) * 4;
+  c->me_threads = me_threads(S);
+  c->me_smem = (size_t)me_smem_words(S) * 4;
 
   std::vector<uint32_t> rank((size_t)S * S), inv((size_t)(S + 1) * (S + 1), 0);
   for (int dy = -c->R; dy < c->R; ++dy)
@@ -127,8 +125,7 @@ extern "C" me_ctx* me_create(int width, int height, int sa_range, int n_rf) {
     c->own_stream = true;
     ok = cudaMemcpy(c->d_rank, rank.data(), rank.size() * 4, cudaMemcpyHostToDevice) == cudaSuccess &&
          cudaMemcpy(c->d_inv, inv.data(), inv.size() * 4, cudaMemcpyHostToDevice) == cudaSuccess &&
-         cudaFuncSetAttribute(me_fsbm_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                              (int)c->me_smem) == cudaSuccess;
+         set_me_smem((int)c->me_smem) == cudaSuccess;
   }
   if (!ok) {
     cudaGetLastError();
@@ -215,11 +212,18 @@ static int launch_me(me_ctx* c, const uint8_t* cf, const uint8_t* const* rfs, in
   P.mb_cols = c->mb_cols; P.row0 = c->row0;
   P.rank_tab = c->d_rank; P.inv_tab = c->d_inv;
   P.out_mvs = mvs; P.out_sads = sads;
-  P.lx = c->lx; P.ngx = c->ngx; P.nsub = c->nsub; P.nwy = c->nwy; P.dyl = c->dyl;
-  P.pw = c->pw; P.cstride = c->cstride;
+  bool vec = (c->W % 16 == 0) && (c->R % 16 == 0);
+  for (int k = 0; k < n_ref; ++k) vec = vec && ((reinterpret_cast<uintptr_t>(rfs[k]) & 15) == 0);
+  P.vec_ok = vec ? 1 : 0;
   dim3 grid(c->mb_cols, c->row1 - c->row0);
   tmark(c, 2, st);
-  me_fsbm_kernel<<<grid, c->me_threads, c->me_smem, st>>>(P);
+  switch (c->S) {   // compile-time window geometry for the paper's SA sizes (Fig. 6a: 32..256)
+    case 16: me_fsbm_kernel<16><<<grid, c->me_threads, c->me_smem, st>>>(P); break;
+    case 32: me_fsbm_kernel<32><<<grid, c->me_threads, c->me_smem, st>>>(P); break;
+    case 64: me_fsbm_kernel<64><<<grid, c->me_threads, c->me_smem, st>>>(P); break;
+    case 128: me_fsbm_kernel<128><<<grid, c->me_threads, c->me_smem, st>>>(P); break;
+    default: me_fsbm_kernel<0><<<grid, c->me_threads, c->me_smem, st>>>(P); break;
+  }
   tmark(c, 3, st);
   c->last_launches++;
   return launch_status();

@@ -41,15 +41,25 @@ struct MeParams {
   const uint32_t* inv_tab;    // rank -> (dx & 0xffff) | (dy << 16)
   int16_t* out_mvs;
   uint16_t* out_sads;
-  int lx, ngx, nsub, nwy, dyl;  // lane / warp geometry (see me_geometry())
-  int pw, cstride;              // shared window: words per row, words per copy
+  int vec_ok;                 // 16-byte aligned rows and window start: vector staging allowed
 };
+
+// ---- launch geometry, shared by host and device (compile-time for the template sizes) ----
+__host__ __device__ constexpr int me_lx(int S) { return S >= 32 ? 32 : S >= 16 ? 16 : S >= 8 ? 8 : 4; }
+__host__ __device__ constexpr int me_ngx(int S) { return (S + me_lx(S) - 1) / me_lx(S); }
+__host__ __device__ constexpr int me_nsub(int S) { return 32 / me_lx(S); }
+__host__ __device__ constexpr int me_dyl(int S) { return ((S + me_nsub(S) - 1) / me_nsub(S) + kMeT - 1) / kMeT * kMeT; }
+__host__ __device__ constexpr int me_pw(int S) { return (((S - 1) >> 2) + 4 + 3) & ~3; }   // words/row, %4 == 0
+__host__ __device__ constexpr int me_cstride(int S) {                                      // == 8 (mod 32)
+  return (S + 15) * me_pw(S) + ((8 - ((S + 15) * me_pw(S)) % 32) % 32 + 32) % 32;
+}
+__host__ __device__ constexpr int me_threads(int S) { return 32 * me_ngx(S); }
+__host__ __device__ constexpr int me_smem_words(int S) { return 64 + 4 * me_cstride(S) + (me_threads(S) / 32) * kNPart; }
 
 // Per-candidate aggregation state carried between 4x4 block rows.
 struct RowState {
-  uint32_t k4prev[4];   // keys of the previous block row's 4x4s
+  uint32_t k4prev[4];   // keys of the previous block row's 4x4s (for 4x8)
   uint32_t p84top[2];   // SADs of the upper 8x4 pair (for 8x8)
-  uint32_t k84top[2];   // keys of the upper 8x4 pair (for 8x8)
   uint32_t p88top[2];   // SADs of the top 8x8 pair (for 8x16)
   uint32_t p168top;     // SAD of the top 16x8 (for 16x16)
 };
@@ -57,41 +67,56 @@ struct RowState {
 constexpr uint32_t kSh = 65536u;
 
 // Keys of every partition completed by 4x4 block row BY of one candidate.
-// L = the four 4x4 SADs of this block row.  Slot -> partition map: part_of().
+// L = the four 4x4 SADs of this block row; key = SAD * 2^16 + rank.  Every key
+// is ONE IMAD (FMA pipe) on a child's SAD or key; plain sums are IMAD.IADD.
+// key(parent) = sad(other child) * 2^16 + key(child): one IMAD.  Written as
+// inline PTX so the compiler cannot re-associate it into add-then-IMAD.
+__device__ __forceinline__ uint32_t kmad(uint32_t sad, uint32_t key) {
+  uint32_t d;
+  asm("mad.lo.u32 %0, %1, 65536, %2;" : "=r"(d) : "r"(sad), "r"(key));
+  return d;
+}
+
+// plain SAD sum kept on the FMA pipe: the ALU pipe is the bottleneck, and an
+// IMAD by an opaque 1 (g_one, a kernel-lifetime register) cannot be fused by
+// ptxas into a 3-input IADD3 on the ALU pipe.
+__device__ __forceinline__ uint32_t fadd(uint32_t a, uint32_t b, uint32_t one) {
+  uint32_t d;
+  asm("mad.lo.u32 %0, %1, %2, %3;" : "=r"(d) : "r"(a), "r"(one), "r"(b));
+  return d;
+}
+
 template <int BY>
 __device__ __forceinline__ void block_row_keys(const uint32_t (&L)[4], uint32_t rank, RowState& st,
-                                               uint32_t (&K)[16]) {
+                                               uint32_t (&K)[16], uint32_t one) {
   uint32_t k4[4];
 #pragma unroll
-  for (int i = 0; i < 4; ++i) k4[i] = L[i] * kSh + rank;
-  const uint32_t p84_0 = L[0] + L[1], p84_1 = L[2] + L[3];
-  const uint32_t k84_0 = L[1] * kSh + k4[0], k84_1 = L[3] * kSh + k4[2];
+  for (int i = 0; i < 4; ++i) k4[i] = kmad(L[i], rank);                   // 4x4
 #pragma unroll
   for (int i = 0; i < 4; ++i) K[i] = k4[i];
-  K[4] = k84_0;
-  K[5] = k84_1;
+  K[4] = kmad(L[1], k4[0]);                                                // 8x4
+  K[5] = kmad(L[3], k4[2]);
+  const uint32_t p84_0 = fadd(L[0], L[1], one), p84_1 = fadd(L[2], L[3], one);
   if ((BY & 1) == 0) {
 #pragma unroll
     for (int i = 0; i < 4; ++i) st.k4prev[i] = k4[i];
     st.p84top[0] = p84_0; st.p84top[1] = p84_1;
-    st.k84top[0] = k84_0; st.k84top[1] = k84_1;
   } else {
 #pragma unroll
-    for (int i = 0; i < 4; ++i) K[6 + i] = L[i] * kSh + st.k4prev[i];      // 4x8
-    const uint32_t k88_0 = p84_0 * kSh + st.k84top[0];                      // 8x8
-    const uint32_t k88_1 = p84_1 * kSh + st.k84top[1];
+    for (int i = 0; i < 4; ++i) K[6 + i] = kmad(L[i], st.k4prev[i]);      // 4x8
+    const uint32_t p88_0 = fadd(p84_0, st.p84top[0], one), p88_1 = fadd(p84_1, st.p84top[1], one);
+    const uint32_t k88_0 = kmad(p88_0, rank), k88_1 = kmad(p88_1, rank);  // 8x8
     K[10] = k88_0;
     K[11] = k88_1;
-    const uint32_t p88_0 = p84_0 + st.p84top[0], p88_1 = p84_1 + st.p84top[1];
-    const uint32_t k168 = p88_1 * kSh + k88_0;                             // 16x8
+    const uint32_t k168 = kmad(p88_1, k88_0);                              // 16x8
     K[12] = k168;
     if (BY == 1) {
       st.p88top[0] = p88_0; st.p88top[1] = p88_1;
-      st.p168top = p88_0 + p88_1;
+      st.p168top = fadd(p88_0, p88_1, one);
     } else {
-      K[13] = st.p88top[0] * kSh + k88_0;                                   // 8x16 left
-      K[14] = st.p88top[1] * kSh + k88_1;                                   // 8x16 right
-      K[15] = st.p168top * kSh + k168;                                      // 16x16
+      K[13] = kmad(st.p88top[0], k88_0);                                    // 8x16 left
+      K[14] = kmad(st.p88top[1], k88_1);                                    // 8x16 right
+      K[15] = kmad(st.p168top, k168);                                       // 16x16
     }
   }
 }
@@ -111,6 +136,7 @@ __host__ __device__ constexpr int part_of(int by, int slot) {
 
 __device__ __forceinline__ uint32_t umin3(uint32_t a, uint32_t b, uint32_t c) { return min(min(a, b), c); }
 
+// fold the keys of a candidate pair into the running minima: one VIMNMX3 per partition
 template <int BY>
 __device__ __forceinline__ void fold_pair(uint32_t (&M)[kNPart], const uint32_t (&Ka)[16], const uint32_t (&Kb)[16]) {
 #pragma unroll
@@ -120,30 +146,43 @@ __device__ __forceinline__ void fold_pair(uint32_t (&M)[kNPart], const uint32_t 
   }
 }
 
-__global__ void __launch_bounds__(256) me_fsbm_kernel(const MeParams P) {
-  extern __shared__ uint32_t smem[];
-  uint32_t* win = smem;                                   // 4 copies x cstride words
-  uint32_t* red = smem + 4 * P.cstride;                   // [nwarps][41]
+// shared-memory loads the compiler may not hoist out of the candidate loop
+// (keeps CF rows out of uniform registers / long-lived registers)
+__device__ __forceinline__ uint4 lds128_v(const uint32_t* p) {
+  uint4 v;
+  const unsigned a = (unsigned)__cvta_generic_to_shared(p);
+  asm volatile("ld.shared.v4.u32 {%0,%1,%2,%3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "r"(a));
+  return v;
+}
+
+// S_CT = compile-time SA size (0 = any even S read from P at run time)
+template <int S_CT>
+__global__ void __launch_bounds__(128, 4) me_fsbm_kernel(const MeParams P) {
+  extern __shared__ __align__(16) uint32_t smem[];
+  const int S = S_CT ? S_CT : P.S;
+  const int R = S / 2;
+  const int PW = me_pw(S), CSTRIDE = me_cstride(S), LX = me_lx(S), NGX = me_ngx(S);
+  const int NSUB = me_nsub(S), DYL = me_dyl(S);
+  uint32_t* cf_s = smem;                                  // 16 rows x 4 words
+  uint32_t* win = smem + 64;                              // 4 copies x CSTRIDE words
+  uint32_t* red = win + 4 * CSTRIDE;                      // [nwarps][41]
 
   const int mbx = blockIdx.x, mby = P.row0 + blockIdx.y;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const uint32_t one = (uint32_t)(P.n_rf > 0);              // == 1, opaque to the compiler (see fadd)
   const int nwarps = blockDim.x >> 5;
-  const int R = P.R, S = P.S;
 
   // ---- lane geometry: dx column and dy sub-range ----
-  const int gx = warp % P.ngx, wyi = warp / P.ngx;
-  const int xi = lane % P.lx, sub = lane / P.lx;
-  const int dx = min(-R + gx * P.lx + xi, R - 1);          // beyond-range lanes duplicate dx=R-1
+  const int gx = warp % NGX;
+  const int xi = lane % LX, sub = lane / LX;
+  const int dx = min(-R + gx * LX + xi, R - 1);            // beyond-range lanes duplicate dx=R-1
   const int off = dx + R;                                  // byte offset inside the window row
-  const uint32_t* wbase = win + (off & 3) * P.cstride + (off >> 2);
-  const int dy_begin = -R + (wyi * P.nsub + sub) * P.dyl;
+  const uint32_t* wbase = win + (off & 3) * CSTRIDE + (off >> 2);
+  const int dy_begin = -R + sub * DYL;
 
-  // ---- CF MB in registers: cf[row][4 words] ----
-  uint32_t cfw[16][4];
-#pragma unroll
-  for (int r = 0; r < 16; ++r)
-#pragma unroll
-    for (int b = 0; b < 4; ++b) cfw[r][b] = load4_clamped(P.cf, P.W, P.H, 16 * mbx + 4 * b, 16 * mby + r);
+  // ---- CF MB -> shared memory (read back as broadcast LDS.128 rows) ----
+  for (int i = threadIdx.x; i < 64; i += blockDim.x)
+    cf_s[i] = load4_clamped(P.cf, P.W, P.H, 16 * mbx + 4 * (i & 3), 16 * mby + (i >> 2));
 
   const int xw0 = 16 * mbx - R, yw0 = 16 * mby - R;
   const int win_rows = S + 15;
@@ -152,15 +191,36 @@ __global__ void __launch_bounds__(256) me_fsbm_kernel(const MeParams P) {
     const uint8_t* __restrict__ rf = P.rf[ref];
     __syncthreads();
     // ---- a1: stage 4 byte-shifted copies of the SA window ----
-    for (int item = threadIdx.x; item < win_rows * P.pw; item += blockDim.x) {
-      const int row = item / P.pw, q = item - row * P.pw;
-      const uint32_t lo = load4_clamped(rf, P.W, P.H, xw0 + 4 * q, yw0 + row);
-      const uint32_t hi = load4_clamped(rf, P.W, P.H, xw0 + 4 * q + 4, yw0 + row);
-      uint32_t* dst = win + row * P.pw + q;
-      dst[0] = lo;
-      dst[P.cstride] = __byte_perm(lo, hi, 0x4321);
-      dst[2 * P.cstride] = __byte_perm(lo, hi, 0x5432);
-      dst[3 * P.cstride] = __byte_perm(lo, hi, 0x6543);
+    // item = (window row, 16-byte chunk k): raw words 4k..4k+4 -> words 4k..4k+3
+    // of copies 0..3 (copy c word q = raw bytes [4q+c, 4q+c+4)), STS.128.
+    {
+      const int chunks = PW >> 2;
+      const bool vec_ok = P.vec_ok;
+      for (int item = threadIdx.x; item < win_rows * chunks; item += blockDim.x) {
+        const int row = item / chunks, k = item - row * chunks;
+        const int x = xw0 + 16 * k, y = min(max(yw0 + row, 0), P.H - 1);
+        uint32_t w[5];
+        if (vec_ok && x >= 0 && x + 20 <= P.W) {
+          const uint8_t* src = rf + (size_t)y * P.W + x;
+          const uint4 v = __ldg(reinterpret_cast<const uint4*>(src));
+          w[0] = v.x; w[1] = v.y; w[2] = v.z; w[3] = v.w;
+          w[4] = __ldg(reinterpret_cast<const uint32_t*>(src + 16));
+        } else {
+#pragma unroll
+          for (int i = 0; i < 5; ++i) w[i] = load4_clamped(rf, P.W, P.H, x + 4 * i, y);
+        }
+        uint32_t* dst = win + row * PW + 4 * k;
+        *reinterpret_cast<uint4*>(dst) = make_uint4(w[0], w[1], w[2], w[3]);
+        *reinterpret_cast<uint4*>(dst + CSTRIDE) =
+            make_uint4(__byte_perm(w[0], w[1], 0x4321), __byte_perm(w[1], w[2], 0x4321),
+                       __byte_perm(w[2], w[3], 0x4321), __byte_perm(w[3], w[4], 0x4321));
+        *reinterpret_cast<uint4*>(dst + 2 * CSTRIDE) =
+            make_uint4(__byte_perm(w[0], w[1], 0x5432), __byte_perm(w[1], w[2], 0x5432),
+                       __byte_perm(w[2], w[3], 0x5432), __byte_perm(w[3], w[4], 0x5432));
+        *reinterpret_cast<uint4*>(dst + 3 * CSTRIDE) =
+            make_uint4(__byte_perm(w[0], w[1], 0x6543), __byte_perm(w[1], w[2], 0x6543),
+                       __byte_perm(w[2], w[3], 0x6543), __byte_perm(w[3], w[4], 0x6543));
+      }
     }
     __syncthreads();
 
@@ -169,33 +229,47 @@ __global__ void __launch_bounds__(256) me_fsbm_kernel(const MeParams P) {
     for (int p = 0; p < kNPart; ++p) M[p] = 0xffffffffu;
 
     const uint32_t* rank_col = P.rank_tab + off;
-    for (int c = 0; c < P.dyl; c += kMeT) {
+    uint32_t rank_next[kMeT];
+    {
+      const int dy0 = min(dy_begin, R - kMeT);
+#pragma unroll
+      for (int t = 0; t < kMeT; ++t) rank_next[t] = __ldg(rank_col + (dy0 + t + R) * S);
+    }
+    for (int c = 0; c < DYL; c += kMeT) {
       const int dy0 = min(dy_begin + c, R - kMeT);        // clamped chunk: duplicates are harmless
       uint32_t rank[kMeT];
 #pragma unroll
-      for (int t = 0; t < kMeT; ++t) rank[t] = __ldg(rank_col + (dy0 + t + R) * S);
-      const uint32_t* wrow = wbase + (dy0 + R) * P.pw;
+      for (int t = 0; t < kMeT; ++t) rank[t] = rank_next[t];
+      {                                                   // prefetch the next chunk's ranks
+        const int dn = min(dy_begin + c + kMeT, R - kMeT);
+#pragma unroll
+        for (int t = 0; t < kMeT; ++t) rank_next[t] = __ldg(rank_col + (dn + t + R) * S);
+      }
+      const uint32_t* wrow = wbase + (dy0 + R) * PW;
 
       uint32_t acc[kMeT][4];
       RowState st[kMeT];
       uint32_t Kp[kMeT][16];
+      uint4 cfr[16];
 #pragma unroll
       for (int i = 0; i < kMeT + 15; ++i) {
+        if (i < 16) cfr[i] = lds128_v(cf_s + 4 * i);     // CF row i, used by RF rows i..i+3
         uint32_t w[4];
 #pragma unroll
-        for (int b = 0; b < 4; ++b) w[b] = wrow[i * P.pw + b];
+        for (int b = 0; b < 4; ++b) w[b] = wrow[i * PW + b];
 #pragma unroll
         for (int t = 0; t < kMeT; ++t) {
           const int r = i - t;                              // CF row paired with RF row i
           if (r >= 0 && r < 16) {
+            const uint32_t cw[4] = {cfr[r].x, cfr[r].y, cfr[r].z, cfr[r].w};
 #pragma unroll
-            for (int b = 0; b < 4; ++b) acc[t][b] = vad4(cfw[r][b], w[b], (r & 3) ? acc[t][b] : 0u);
+            for (int b = 0; b < 4; ++b) acc[t][b] = vad4(cw[b], w[b], (r & 3) ? acc[t][b] : 0u);
             if ((r & 3) == 3) {
               const int by = r >> 2;
-              if (by == 0) block_row_keys<0>(acc[t], rank[t], st[t], Kp[t]);
-              if (by == 1) block_row_keys<1>(acc[t], rank[t], st[t], Kp[t]);
-              if (by == 2) block_row_keys<2>(acc[t], rank[t], st[t], Kp[t]);
-              if (by == 3) block_row_keys<3>(acc[t], rank[t], st[t], Kp[t]);
+              if (by == 0) block_row_keys<0>(acc[t], rank[t], st[t], Kp[t], one);
+              if (by == 1) block_row_keys<1>(acc[t], rank[t], st[t], Kp[t], one);
+              if (by == 2) block_row_keys<2>(acc[t], rank[t], st[t], Kp[t], one);
+              if (by == 3) block_row_keys<3>(acc[t], rank[t], st[t], Kp[t], one);
               if (t & 1) {                                  // pair (t-1, t) finished this block row
                 if (by == 0) fold_pair<0>(M, Kp[t - 1], Kp[t]);
                 if (by == 1) fold_pair<1>(M, Kp[t - 1], Kp[t]);
