@@ -241,12 +241,26 @@ static int launch_int(me_ctx* c, const uint8_t* rf, uint8_t* sf, cudaStream_t st
     P.row_end = std::min(c->sf_rows, c->sf_pad + 16 * c->row1 + c->R + 4);
   }
   const int groups = c->sf_pitch / 16;
+  // interior groups: x0-4 >= 0 and x0+20 <= W with x0 = 16g - pad, rows 4-byte aligned
+  int g_lo = groups, g_hi = groups;
+  if (c->W % 4 == 0 && (reinterpret_cast<uintptr_t>(rf) & 3) == 0) {
+    g_lo = std::min(groups, (c->sf_pad + 4 + 15) / 16);
+    g_hi = std::max(g_lo, std::min(groups, (c->W - 20 + c->sf_pad) / 16 + 1));
+  }
+  P.g_lo = g_lo; P.g_hi = g_hi;
   dim3 block(32, 4);
-  dim3 grid((groups + 31) / 32, (P.row_end - P.row_begin + 3) / 4);
+  const int nrows = P.row_end - P.row_begin;
   tmark(c, 0, st);
-  int_subpel_kernel<<<grid, block, 0, st>>>(P);
+  if (g_hi > g_lo) {
+    int_subpel_kernel<true><<<dim3((g_hi - g_lo + 31) / 32, (nrows + 3) / 4), block, 0, st>>>(P);
+    c->last_launches++;
+  }
+  const int nb = groups - (g_hi - g_lo);
+  if (nb > 0) {
+    int_subpel_kernel<false><<<dim3((nb + 31) / 32, (nrows + 3) / 4), block, 0, st>>>(P);
+    c->last_launches++;
+  }
   tmark(c, 1, st);
-  c->last_launches++;
   return launch_status();
 }
 
@@ -261,12 +275,13 @@ static int launch_sme(me_ctx* c, const uint8_t* cf, const uint8_t* const* sfs, c
   P.out_qmvs = reinterpret_cast<uint32_t*>(out_qmvs);
   P.out_sads = out_sads;
   P.W = c->W; P.H = c->H; P.n_rf = n_ref; P.rf_stride = c->n_rf; P.mb_cols = c->mb_cols; P.row0 = c->row0;
-  P.n_items = (c->row1 - c->row0) * c->mb_cols * n_ref;
+  P.n_rows = c->row1 - c->row0;
+  P.groups = (c->mb_cols + 7) / 8;
   P.pad = c->sf_pad; P.pitch = c->sf_pitch;
   P.plane = (size_t)c->sf_rows * c->sf_pitch;
-  const int per_block = 128 / 16;
+  const int warps = n_ref * P.n_rows * P.groups;
   tmark(c, 4, st);
-  sme_refine_kernel<<<(P.n_items + per_block - 1) / per_block, 128, 0, st>>>(P);
+  sme_refine_kernel<<<(warps + 3) / 4, 128, 0, st>>>(P);
   tmark(c, 5, st);
   c->last_launches++;
   return launch_status();

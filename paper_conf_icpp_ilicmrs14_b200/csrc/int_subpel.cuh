@@ -6,12 +6,14 @@
 // Filter (O2, the H.264 luma interpolation the paper inherits via
 // JM 18.4): tap (1,-5,20,20,-5,1); b,h,m,s = Clip1((x1+16)>>5);
 // j = Clip1((j1+512)>>10) with j1 taken horizontally over h1 (equal to the
-// vertical form, pin P6); the 12 quarter samples are (u+v+1)>>1 averages,
-// done four at a time with VAVRG4.
+// vertical form, pin P6); the 12 quarter samples are (u+v+1)>>1 averages.
 //
-// One thread = 16 consecutive plane columns of one plane row; a warp writes
-// 32 x 16 B = 512 contiguous bytes per plane with 128-bit stores (HBM-bound
-// kernel: 1 B read + 16 B written per position).
+// One thread = 16 consecutive plane columns of one plane row.  The 6-tap
+// filters on b1/h1/s1 (range [-2550, 10710]) run two columns per 32-bit
+// instruction on biased, non-negative 16-bit lanes (plain IADD / IMAD by 20
+// and -5, exact per lane); j1 (20-bit) runs in int32.  Quarter samples: VAVRG4 on 4 packed
+// bytes.  A warp writes 32 x 16 B = 512 contiguous bytes per plane with
+// 128-bit stores (HBM-bound kernel: 1 B read + 16 B written per position).
 #pragma once
 #include "common.cuh"
 
@@ -22,64 +24,113 @@ struct IntParams {
   uint8_t* sf;
   int W, H, pad, pitch, rows, row_begin, row_end;
   size_t plane;   // bytes per phase plane = rows * pitch
+  int g_lo, g_hi; // interior 16-column groups [g_lo, g_hi): every source word in-frame and aligned
 };
 
-__device__ __forceinline__ int tap6(int a, int b, int c, int d, int e, int f) {
-  return (a + f) - 5 * (b + e) + 20 * (c + d);
+// Two columns per 32-bit register, one per 16-bit lane, and every lane kept
+// NON-NEGATIVE so plain 32-bit IADD/IMAD are exact per lane (no carry or
+// borrow can cross lanes).  A 6-tap result x1 in [-2550, 10710] is carried as
+// x1 + 2560 in [10, 13270]; 2560 = 80 * 32 cancels exactly in the >>5 and
+// >>10 roundings.  (No 16x2 subtraction: ptxas was seen to
+// miscompile __vsub2 when one lane is dead.)
+constexpr uint32_t kBias = 2560u;
+constexpr uint32_t kBias2 = kBias | (kBias << 16);
+// tap6 on packed byte columns: (a+f) - 5(b+e) + 20(c+d) + 2560, per lane
+__device__ __forceinline__ uint32_t tap6x2b(uint32_t a, uint32_t b, uint32_t c, uint32_t d, uint32_t e, uint32_t f) {
+  const uint32_t s = a + f, q = b + e, m = c + d;                   // lanes <= 510: no carry
+  return (m * 20u + s) + (kBias2 - q * 5u);                          // lanes in [10, 13270]
 }
-__device__ __forceinline__ uint32_t clip255(int v) { return (uint32_t)min(max(v, 0), 255); }
-
-__device__ __forceinline__ uint32_t pack4(uint32_t a, uint32_t b, uint32_t c, uint32_t d) {
-  return __byte_perm(__byte_perm(a, b, 0x0040), __byte_perm(c, d, 0x0040), 0x5410);
+// Clip1((x1 + 16) >> 5) on two biased lanes -> two u16 lanes in [0, 255]
+__device__ __forceinline__ uint32_t clip_half2(uint32_t vb) {
+  const uint32_t t = ((vb + 0x00100010u) >> 5) & 0x07ff07ffu;       // ((x1+16)>>5) + 80 per lane
+  return __vminu2(__vmaxu2(t, 0x00500050u), 0x014f014fu) - 0x00500050u;   // clamp to [80, 335], -80
 }
+__device__ __forceinline__ int lo_u16(uint32_t x) { return (int)(x & 0xffffu); }
+__device__ __forceinline__ int hi_u16(uint32_t x) { return (int)(x >> 16); }
+// j = Clip1((j1 + 512) >> 10) from the biased sum jb = j1 + 32 * 2560
+__device__ __forceinline__ uint32_t clip_j(int jb) { return (uint32_t)min(max(jb - (32 * (int)kBias - 512), 0) >> 10, 255); }
 
+// low bytes of four u16 lanes (pairs a, b) -> one byte word
+__device__ __forceinline__ uint32_t bytes_of(uint32_t a, uint32_t b) { return __byte_perm(a, b, 0x6420); }
+
+// INTERIOR launch: groups [g_lo, g_hi) (no clamping code at all, warps never
+// diverge); border launch: the groups outside it, with per-byte clamping.
+template <bool INTERIOR>
 __global__ void __launch_bounds__(128) int_subpel_kernel(const IntParams P) {
-  const int g = blockIdx.x * blockDim.x + threadIdx.x;    // 16-column group
+  const int t = blockIdx.x * blockDim.x + threadIdx.x;
+  const int nb_left = P.g_lo;
+  const int g = INTERIOR ? P.g_lo + t : (t < nb_left ? t : P.g_hi + (t - nb_left));   // 16-column group
   const int rr = P.row_begin + blockIdx.y * blockDim.y + threadIdx.y;
-  if (16 * g >= P.pitch || rr >= P.row_end) return;
+  if ((INTERIOR ? g >= P.g_hi : 16 * g >= P.pitch) || rr >= P.row_end) return;
   const int x0 = 16 * g - P.pad, y = rr - P.pad;
 
-  // source rows y-2 .. y+3, columns x0-4 .. x0+19 (6 words per row)
+  // source rows y-2 .. y+3 (k = 0..5), columns x0-4 .. x0+19 (c = 0..23, 6 words)
   uint32_t w[6][6];
 #pragma unroll
-  for (int k = 0; k < 6; ++k)
+  for (int k = 0; k < 6; ++k) {
+    const int yy = clampi(y - 2 + k, 0, P.H - 1);
+    if (INTERIOR) {
+      const uint32_t* src = reinterpret_cast<const uint32_t*>(P.rf + (size_t)yy * P.W + x0 - 4);
 #pragma unroll
-    for (int q = 0; q < 6; ++q) w[k][q] = load4_clamped(P.rf, P.W, P.H, x0 - 4 + 4 * q, y - 2 + k);
-  auto px = [&](int k, int c) -> int { return (int)((w[k][c >> 2] >> (8 * (c & 3))) & 0xffu); };  // c: col - (x0-4)
+      for (int q = 0; q < 6; ++q) w[k][q] = __ldg(src + q);
+    } else {
+#pragma unroll
+      for (int q = 0; q < 6; ++q) w[k][q] = load4_clamped(P.rf, P.W, P.H, x0 - 4 + 4 * q, yy);
+    }
+  }
+  // byte pairs as u16x2: pr[k][j] = columns (2j, 2j+1)
+  auto pr = [&](int k, int j) -> uint32_t { return __byte_perm(w[k][j >> 1], 0, (j & 1) ? 0x4342 : 0x4140); };
 
-  // h1 at columns x0-2 .. x0+18 (index j <-> column x0-2+j), vertical taps
-  int h1[21];
+  // h1 on columns c = 2..23 (pairs j = 1..11), vertical taps
+  uint32_t h1[12];
 #pragma unroll
-  for (int j = 0; j < 21; ++j)
-    h1[j] = tap6(px(0, j + 2), px(1, j + 2), px(2, j + 2), px(3, j + 2), px(4, j + 2), px(5, j + 2));
+  for (int j = 1; j < 12; ++j) h1[j] = tap6x2b(pr(0, j), pr(1, j), pr(2, j), pr(3, j), pr(4, j), pr(5, j));
+
+  // b1 (row k=2) and s1 (row k=3) at output columns c = 4..19 (pairs j = 2..9), horizontal taps
+  uint32_t bc[8], sc[8];
+#pragma unroll
+  for (int k = 2; k <= 3; ++k) {
+    uint32_t p[12];
+#pragma unroll
+    for (int j = 1; j < 12; ++j) p[j] = pr(k, j);
+#pragma unroll
+    for (int j = 2; j < 10; ++j) {
+      const uint32_t xm1 = __byte_perm(p[j - 1], p[j], 0x5432);     // columns (2j-1, 2j)
+      const uint32_t xp1 = __byte_perm(p[j], p[j + 1], 0x5432);     // (2j+1, 2j+2)
+      const uint32_t xp3 = __byte_perm(p[j + 1], p[j + 2], 0x5432); // (2j+3, 2j+4)
+      const uint32_t v = clip_half2(tap6x2b(p[j - 1], xm1, p[j], xp1, p[j + 1], xp3));
+      if (k == 2) bc[j - 2] = v; else sc[j - 2] = v;
+    }
+  }
+  // h and m = h at x+1: clipped h1 on pairs j = 2..10 (columns 4..21)
+  uint32_t hc[9];
+#pragma unroll
+  for (int j = 2; j < 11; ++j) hc[j - 2] = clip_half2(h1[j]);
+
+  // j1 = tap6 over h1 at columns c-2..c+3 (int32), c = 4..19
+  int hv[22];
+#pragma unroll
+  for (int j = 1; j < 12; ++j) { hv[2 * j - 2] = lo_u16(h1[j]); hv[2 * j - 1] = hi_u16(h1[j]); }   // hv[i] = h1 + 2560 at c = i+2
+  uint32_t jb[16];
+#pragma unroll
+  for (int i = 0; i < 16; ++i) {   // output column c = i+4: h1 at c-2..c+3 = hv[i .. i+5]
+    const int j1 = (hv[i] + hv[i + 5]) - 5 * (hv[i + 1] + hv[i + 4]) + 20 * (hv[i + 2] + hv[i + 3]);
+    jb[i] = clip_j(j1);
+  }
 
   uint32_t Gw[4], Hw[4], Mw[4], bw[4], hw[4], mw[4], sw[4], jw[4];
 #pragma unroll
   for (int q = 0; q < 4; ++q) {
-    uint32_t G[4], Hh[4], M[4], b[4], h[4], m[4], s[4], j[4];
-#pragma unroll
-    for (int u = 0; u < 4; ++u) {
-      const int i = 4 * q + u;                 // position x0 + i; row-2 column index i+4
-      G[u] = px(2, i + 4);
-      Hh[u] = px(2, i + 5);
-      M[u] = px(3, i + 4);
-      const int b1 = tap6(px(2, i + 2), px(2, i + 3), px(2, i + 4), px(2, i + 5), px(2, i + 6), px(2, i + 7));
-      const int s1 = tap6(px(3, i + 2), px(3, i + 3), px(3, i + 4), px(3, i + 5), px(3, i + 6), px(3, i + 7));
-      const int j1 = tap6(h1[i], h1[i + 1], h1[i + 2], h1[i + 3], h1[i + 4], h1[i + 5]);
-      b[u] = clip255((b1 + 16) >> 5);
-      s[u] = clip255((s1 + 16) >> 5);
-      h[u] = clip255((h1[i + 2] + 16) >> 5);
-      m[u] = clip255((h1[i + 3] + 16) >> 5);
-      j[u] = clip255((j1 + 512) >> 10);
-    }
-    Gw[q] = pack4(G[0], G[1], G[2], G[3]);
-    Hw[q] = pack4(Hh[0], Hh[1], Hh[2], Hh[3]);
-    Mw[q] = pack4(M[0], M[1], M[2], M[3]);
-    bw[q] = pack4(b[0], b[1], b[2], b[3]);
-    hw[q] = pack4(h[0], h[1], h[2], h[3]);
-    mw[q] = pack4(m[0], m[1], m[2], m[3]);
-    sw[q] = pack4(s[0], s[1], s[2], s[3]);
-    jw[q] = pack4(j[0], j[1], j[2], j[3]);
+    Gw[q] = w[2][q + 1];                                        // columns 4q+4 .. 4q+7
+    Hw[q] = __funnelshift_r(w[2][q + 1], w[2][q + 2], 8);       // +1 column
+    Mw[q] = w[3][q + 1];                                        // row y+1
+    bw[q] = bytes_of(bc[2 * q], bc[2 * q + 1]);
+    sw[q] = bytes_of(sc[2 * q], sc[2 * q + 1]);
+    hw[q] = bytes_of(hc[2 * q], hc[2 * q + 1]);
+    // m: columns 4q+5..4q+8 = hc[2q] hi, hc[2q+1] lo/hi, hc[2q+2] lo
+    mw[q] = __byte_perm(bytes_of(hc[2 * q], hc[2 * q + 1]), bytes_of(hc[2 * q + 2], hc[2 * q + 2]), 0x4321);
+    jw[q] = __byte_perm(__byte_perm(jb[4 * q], jb[4 * q + 1], 0x0040), __byte_perm(jb[4 * q + 2], jb[4 * q + 3], 0x0040),
+                        0x5410);
   }
 
   uint8_t* dst = P.sf + (size_t)rr * P.pitch + 16 * g;

@@ -7,12 +7,14 @@
 // stage: the 8 ring-1 neighbours c + 2*s_k in spiral order, update on strict
 // <; quarter stage: the 8 neighbours of the best half position, strict <.
 //
-// 16 lanes = the 16 4x4 blocks of one (MB, RF).  Lane bits (bx0, by0, bx1,
-// by1) make every partition of every mode an xor-closed lane set, so each
-// partition's SAD is a butterfly all-reduce over that mode's bits and every
-// lane of a partition holds the same (best, bestv) -- no divergence.  Each
-// lane computes, per mode and candidate, the SAD of its own 4x4 block against
-// the SF phase plane (4 rows x one unaligned 4-byte window, VABSDIFF4.ACC).
+// Mapping (L1-sector bound kernel): one warp = 8 horizontally
+// adjacent MBs of one RF x 4 lanes; lane (g, bx) owns the 4-pixel column
+// strip bx of MB g (its four 4x4 blocks by = 0..3, CF strip in 16 registers).
+// For one candidate, every LDG of the warp reads one row of 8 x 16 contiguous
+// bytes of one SF phase plane when the MBs' MVs agree (the common case), so a
+// request touches ~5 sectors instead of 16.  A partition's SAD = sum over its
+// blocks: inside the lane over by, across lanes by xor-shuffles over bx bits;
+// every lane of a partition then holds the same (best, bestv) -- no divergence.
 #pragma once
 #include "common.cuh"
 
@@ -25,20 +27,20 @@ struct SmeParams {
   const uint16_t* in_sads;    // may be null
   uint32_t* out_qmvs;
   uint16_t* out_sads;
-  int W, H, n_rf, rf_stride, mb_cols, row0, n_items;   // n_rf RFs refined, rf_stride = layout
+  int W, H, n_rf, rf_stride, mb_cols, row0, n_rows;   // n_rf RFs refined, rf_stride = layout
+  int groups;                                         // ceil(mb_cols / 8)
   int pad, pitch;
   size_t plane;
 };
 
-__constant__ int8_t c_ring1[8][2] = {{0, -1}, {0, 1}, {-1, -1}, {1, -1}, {-1, 0}, {1, 0}, {-1, 1}, {1, 1}};
+// ring-1 spiral order s_k (G12/G14), compile-time so unrolled loops fold it
+__device__ constexpr int8_t c_ring1[8][2] = {{0, -1}, {0, 1}, {-1, -1}, {1, -1}, {-1, 0}, {1, 0}, {-1, 1}, {1, 1}};
 
-// 4x4 SAD of this lane's CF block against SF samples at quarter-pel offset v
-__device__ __forceinline__ uint32_t block_sad_q(const uint8_t* __restrict__ sf, size_t plane, int pitch,
-                                                int pad, int bxp, int byp, int vx, int vy,
-                                                const uint32_t (&cfb)[4]) {
+// SAD of this lane's 4x4 block (rows ys..ys+3 of the strip) vs SF samples at quarter offset v
+__device__ __forceinline__ uint32_t strip_block_sad(const uint8_t* __restrict__ sf, size_t plane, int pitch, int pad,
+                                                    int xs, int ys, int vx, int vy, const uint32_t* cfr) {
   const uint8_t* pl = sf + (size_t)(4 * (vy & 3) + (vx & 3)) * plane;
-  const int X = bxp + (vx >> 2) + pad, Y = byp + (vy >> 2) + pad;
-  const uint8_t* p0 = pl + (size_t)Y * pitch + X;
+  const uint8_t* p0 = pl + (size_t)(ys + (vy >> 2) + pad) * pitch + (xs + (vx >> 2) + pad);
   const uintptr_t a = reinterpret_cast<uintptr_t>(p0);
   const uint32_t* w = reinterpret_cast<const uint32_t*>(a & ~uintptr_t(3));
   const uint32_t sh = 8u * (uint32_t)(a & 3);
@@ -47,72 +49,125 @@ __device__ __forceinline__ uint32_t block_sad_q(const uint8_t* __restrict__ sf, 
 #pragma unroll
   for (int r = 0; r < 4; ++r) {
     const uint32_t lo = __ldg(w + r * wp), hi = __ldg(w + r * wp + 1);
-    s = vad4(cfb[r], __funnelshift_r(lo, hi, sh), s);
+    s = vad4(cfr[r], __funnelshift_r(lo, hi, sh), s);
   }
   return s;
 }
 
-// all-reduce over the xor-closed lane set of one partition (offsets < 16 stay
-// inside the 16-lane half that owns this (MB, RF))
-template <int MASK>
-__device__ __forceinline__ uint32_t part_sum(uint32_t v) {
-  const unsigned half = (threadIdx.x & 16) ? 0xffff0000u : 0x0000ffffu;
-  if (MASK & 1) v += __shfl_xor_sync(half, v, 1);
-  if (MASK & 2) v += __shfl_xor_sync(half, v, 2);
-  if (MASK & 4) v += __shfl_xor_sync(half, v, 4);
-  if (MASK & 8) v += __shfl_xor_sync(half, v, 8);
+template <int XMASK>
+__device__ __forceinline__ uint32_t xsum(uint32_t v) {   // all-reduce over the bx lane bits in XMASK
+  if (XMASK & 1) v += __shfl_xor_sync(0xffffffffu, v, 1);
+  if (XMASK & 2) v += __shfl_xor_sync(0xffffffffu, v, 2);
   return v;
 }
 
-template <int MASK>
-__device__ __forceinline__ void refine_mode(const SmeParams& P, const uint8_t* __restrict__ sf, int p, size_t o,
-                                            int bxp, int byp, int b, const uint32_t (&cfb)[4]) {
-  const uint32_t mv = __ldg(P.in_mvs + o + p);
-  const int cx = 4 * (int)(int16_t)(mv & 0xffffu), cy = 4 * (int)(int16_t)(mv >> 16);
-  uint32_t best = P.in_sads ? (uint32_t)__ldg(P.in_sads + o + p)
-                            : part_sum<MASK>(block_sad_q(sf, P.plane, P.pitch, P.pad, bxp, byp, cx, cy, cfb));
-  int bvx = cx, bvy = cy;
-#pragma unroll
-  for (int k = 0; k < 8; ++k) {              // half-pel ring around c
-    const int vx = cx + 2 * c_ring1[k][0], vy = cy + 2 * c_ring1[k][1];
-    const uint32_t s = part_sum<MASK>(block_sad_q(sf, P.plane, P.pitch, P.pad, bxp, byp, vx, vy, cfb));
-    if (s < best) { best = s; bvx = vx; bvy = vy; }
+// partition index (G7) of block (bx, by) in each mode
+template <int MODE>
+__device__ __forceinline__ int mode_part(int bx, int by) {
+  const int s = 2 * (by >> 1) + (bx >> 1);
+  switch (MODE) {
+    case 0: return 0;                                      // 16x16
+    case 1: return 1 + (by >> 1);                          // 16x8
+    case 2: return 3 + (bx >> 1);                          // 8x16
+    case 3: return 5 + s;                                  // 8x8
+    case 4: return 9 + 2 * s + (by & 1);                   // 8x4 (w8 h4)
+    case 5: return 17 + 2 * s + (bx & 1);                  // 4x8 (w4 h8)
+    default: return 25 + 4 * s + 2 * (by & 1) + (bx & 1);  // 4x4
   }
-  const int hx = bvx, hy = bvy;
+}
+
+// YG = blocks of a partition along by inside the lane (1, 2, 4);
+// XMASK = the bx lane bits a partition spans (0, 1, 3).
+template <int MODE, int YG, int XMASK>
+__device__ __forceinline__ void refine_mode(const SmeParams& P, const uint8_t* __restrict__ sf, size_t o, int bx,
+                                            int xs, int ys0, bool writer, const uint32_t (&cfs)[16]) {
+  constexpr int NG = 4 / YG;           // partitions (block groups) inside this lane's strip
+  int bvx[NG], bvy[NG];
+  uint32_t best[NG];
 #pragma unroll
-  for (int k = 0; k < 8; ++k) {              // quarter-pel ring around the best half position
-    const int vx = hx + c_ring1[k][0], vy = hy + c_ring1[k][1];
-    const uint32_t s = part_sum<MASK>(block_sad_q(sf, P.plane, P.pitch, P.pad, bxp, byp, vx, vy, cfb));
-    if (s < best) { best = s; bvx = vx; bvy = vy; }
+  for (int g = 0; g < NG; ++g) {
+    const int p = mode_part<MODE>(bx, g * YG);
+    const uint32_t mv = __ldg(P.in_mvs + o + p);
+    bvx[g] = 4 * (int)(int16_t)(mv & 0xffffu);
+    bvy[g] = 4 * (int)(int16_t)(mv >> 16);
+    if (P.in_sads) {
+      best[g] = __ldg(P.in_sads + o + p);
+    } else {
+      uint32_t s = 0;
+#pragma unroll
+      for (int j = 0; j < YG; ++j)
+        s += strip_block_sad(sf, P.plane, P.pitch, P.pad, xs, ys0 + 4 * (g * YG + j), bvx[g], bvy[g],
+                             cfs + 4 * (g * YG + j));
+      best[g] = xsum<XMASK>(s);
+    }
   }
-  if ((b & MASK) == 0) {                     // partition leader writes
-    P.out_qmvs[o + p] = (uint32_t)(uint16_t)bvx | ((uint32_t)(uint16_t)bvy << 16);
-    P.out_sads[o + p] = (uint16_t)best;
+#pragma unroll
+  for (int stage = 0; stage < 2; ++stage) {
+    int ox[NG], oy[NG];
+#pragma unroll
+    for (int g = 0; g < NG; ++g) { ox[g] = bvx[g]; oy[g] = bvy[g]; }   // half: c; quarter: best half
+    // all 8 ring candidates' loads first (memory-level parallelism: the kernel
+    // is latency-bound), then the strictly ordered compare/updates
+    uint32_t sad[8][NG];
+#pragma unroll
+    for (int k = 0; k < 8; ++k) {
+      const int sx = c_ring1[k][0] << (1 - stage), sy = c_ring1[k][1] << (1 - stage);
+#pragma unroll
+      for (int g = 0; g < NG; ++g) {
+        uint32_t t = 0;
+#pragma unroll
+        for (int j = 0; j < YG; ++j)
+          t += strip_block_sad(sf, P.plane, P.pitch, P.pad, xs, ys0 + 4 * (g * YG + j), ox[g] + sx, oy[g] + sy,
+                               cfs + 4 * (g * YG + j));
+        sad[k][g] = t;
+      }
+    }
+#pragma unroll
+    for (int k = 0; k < 8; ++k) {
+      const int sx = c_ring1[k][0] << (1 - stage), sy = c_ring1[k][1] << (1 - stage);
+#pragma unroll
+      for (int g = 0; g < NG; ++g) {
+        const uint32_t t = xsum<XMASK>(sad[k][g]);
+        if (t < best[g]) { best[g] = t; bvx[g] = ox[g] + sx; bvy[g] = oy[g] + sy; }
+      }
+    }
+  }
+  if (writer && (bx & XMASK) == 0) {     // partition leader lane writes
+#pragma unroll
+    for (int g = 0; g < NG; ++g) {
+      const int p = mode_part<MODE>(bx, g * YG);
+      P.out_qmvs[o + p] = (uint32_t)(uint16_t)bvx[g] | ((uint32_t)(uint16_t)bvy[g] << 16);
+      P.out_sads[o + p] = (uint16_t)best[g];
+    }
   }
 }
 
 __global__ void __launch_bounds__(128) sme_refine_kernel(const SmeParams P) {
-  const int item = blockIdx.x * (blockDim.x >> 4) + (threadIdx.x >> 4);
-  if (item >= P.n_items) return;             // whole 16-lane groups exit together
-  const int b = threadIdx.x & 15;
-  const int bx0 = b & 1, by0 = (b >> 1) & 1, bx1 = (b >> 2) & 1, by1 = (b >> 3) & 1;
-  const int bx = 2 * bx1 + bx0, by = 2 * by1 + by0;
-  const int ref = item % P.n_rf, mbi = item / P.n_rf;
-  const int mbx = mbi % P.mb_cols, mby = P.row0 + mbi / P.mb_cols;
-  const int bxp = 16 * mbx + 4 * bx, byp = 16 * mby + 4 * by;
-  uint32_t cfb[4];
+  const int warp_id = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
+  const int n_warps = P.n_rf * P.n_rows * P.groups;
+  if (warp_id >= n_warps) return;                    // whole warps exit together
+  const int lane = threadIdx.x & 31;
+  const int gi = warp_id % P.groups;
+  const int rem = warp_id / P.groups;
+  const int mrow = rem % P.n_rows, ref = rem / P.n_rows;
+  const int bx = lane & 3;
+  const int mbx_raw = 8 * gi + (lane >> 2);
+  const bool writer = mbx_raw < P.mb_cols;
+  const int mbx = min(mbx_raw, P.mb_cols - 1);       // surplus lanes duplicate the last MB
+  const int mby = P.row0 + mrow;
+  const int xs = 16 * mbx + 4 * bx, ys0 = 16 * mby;
+  uint32_t cfs[16];
 #pragma unroll
-  for (int r = 0; r < 4; ++r) cfb[r] = load4_clamped(P.cf, P.W, P.H, bxp, byp + r);
+  for (int r = 0; r < 16; ++r) cfs[r] = load4_clamped(P.cf, P.W, P.H, xs, ys0 + r);
   const uint8_t* __restrict__ sf = P.sf[ref];
-  const size_t o = ((size_t)mbi * P.rf_stride + ref) * kNPart;    // [mb][ref][41]
-  const int s = 2 * by1 + bx1;
-  refine_mode<15>(P, sf, 0, o, bxp, byp, b, cfb);                           // 16x16
-  refine_mode<7>(P, sf, 1 + by1, o, bxp, byp, b, cfb);                      // 16x8
-  refine_mode<11>(P, sf, 3 + bx1, o, bxp, byp, b, cfb);                     // 8x16
-  refine_mode<3>(P, sf, 5 + s, o, bxp, byp, b, cfb);                        // 8x8
-  refine_mode<1>(P, sf, 9 + 2 * s + by0, o, bxp, byp, b, cfb);              // 8x4
-  refine_mode<2>(P, sf, 17 + 2 * s + bx0, o, bxp, byp, b, cfb);             // 4x8
-  refine_mode<0>(P, sf, 25 + 4 * s + 2 * by0 + bx0, o, bxp, byp, b, cfb);   // 4x4
+  const size_t o = ((size_t)(mrow * P.mb_cols + mbx) * P.rf_stride + ref) * kNPart;
+  refine_mode<0, 4, 3>(P, sf, o, bx, xs, ys0, writer, cfs);   // 16x16
+  refine_mode<1, 2, 3>(P, sf, o, bx, xs, ys0, writer, cfs);   // 16x8
+  refine_mode<2, 4, 1>(P, sf, o, bx, xs, ys0, writer, cfs);   // 8x16
+  refine_mode<3, 2, 1>(P, sf, o, bx, xs, ys0, writer, cfs);   // 8x8
+  refine_mode<4, 1, 1>(P, sf, o, bx, xs, ys0, writer, cfs);   // 8x4
+  refine_mode<5, 2, 0>(P, sf, o, bx, xs, ys0, writer, cfs);   // 4x8
+  refine_mode<6, 1, 0>(P, sf, o, bx, xs, ys0, writer, cfs);   // 4x4
 }
 
 }  // namespace feves
