@@ -285,14 +285,28 @@ def run_feves(args, cfg):
     int_iso_ms = statistics.mean(a.elapsed_time(b) for a, b in iso)
     del sf_scratch
 
+    # ME alone (no SME), the kernel the roofline names, in the same launch configuration
+    me_only = []
+    mvs_scratch = me.new_mvs()
+    rf_list = [frames[(t - 1 - k) % n_frames] for k in range(cfg.n_rf)]
+    for k in range(max(3, min(args.steps, 20))):
+        flush.fill_(k & 0xff)
+        me.estimate(frames[t % n_frames], rf_list, out=mvs_scratch)
+        me_only.append(me.timings()[1])
+    del mvs_scratch
+
     u = workload_units(cfg)
     int_ms = statistics.mean(m[0] for m in mod)
-    me_ms = statistics.mean(m[1] for m in mod)
-    sme_ms = statistics.mean(m[2] for m in mod)
+    fused = all(m[2] < 0 for m in mod)
+    me_ms = statistics.mean(m[1] for m in mod)              # fused: ME + SME in one kernel
+    sme_ms = None if fused else statistics.mean(m[2] for m in mod)
+    me_only_ms = statistics.mean(me_only)
     stripe_frac = (r1 - r0) / me.mb_rows
     pk, pk_src = peaks()
     peak_px = N_SM * PX_PER_CLK_SM * pk.get("sm_max_mhz", 1965.0) * 1e6
-    achieved_px = u["me_px"] * stripe_frac / (me_ms / 1e3)
+    dom_px = (u["me_px"] + (u["sme_px"] if fused else 0)) * stripe_frac
+    achieved_px = dom_px / (me_ms / 1e3)
+    me_only_px = u["me_px"] * stripe_frac / (me_only_ms / 1e3)
     traffic = None
     try:
         with open(os.path.join(ROOT, "profiles", "ncu_traffic.json")) as f:
@@ -338,19 +352,26 @@ def run_feves(args, cfg):
         "config": config_json(cfg, args),
         "candidate_gsad_per_s": u["gsad"] * fps / 1e9,
         "px_absdiff_per_s": (u["me_px"] + u["sme_px"]) * fps,
-        "kernels_ms": {"int_in_step": int_ms, "me": me_ms, "sme": sme_ms, "int_isolated": int_iso_ms,
-                       "note": "CUDA events around each launch on its own stream; in the step INT runs "
-                               "concurrently with ME (P:86), so int_in_step includes sharing the SMs with ME"},
+        "kernels_ms": {"int": int_ms, ("me_sme_fused" if fused else "me"): me_ms, "sme": sme_ms,
+                       "int_isolated": int_iso_ms, "me_only_isolated": me_only_ms,
+                       "note": "CUDA events around each launch on its own stream" + (
+                           "; fused: INT(t-1) then one ME+SME kernel" if fused else
+                           "; INT runs concurrently with ME (P:86) on a side stream")},
         "clocks": ck,
         "e2e": e2e,
         "gpu_launches": launches,
-        "roofline": {"bound": "alu", "kernel": "me_fsbm_kernel", "achieved": achieved_px / 1e12,
+        "roofline": {"bound": "alu", "kernel": "me_fsbm_kernel<64,fused>" if fused else "me_fsbm_kernel<64>",
+                     "work": "px-absdiffs of ME" + (" + SME (fused kernel)" if fused else "") + " per launch",
+                     "achieved": achieved_px / 1e12,
                      "peak": peak_px / 1e12, "unit": "Tpx-absdiff/s", "frac": achieved_px / peak_px,
                      "traffic": traffic,
                      "peak_source": f"148 SM x 64 VABSDIFF4 lanes/clk x 4 px x sm_max_mhz ({pk_src} "
                                     "MEASURED_PEAKS.json); issue rate measured in profiles/r01/int_peaks.json",
                      "frac_at_observed_clock": (achieved_px / (N_SM * PX_PER_CLK_SM * ck["sm_mhz"] * 1e6))
                      if ck.get("sm_mhz") else None},
+        "roofline_me_only": {"bound": "alu", "kernel": "me_fsbm_kernel<64> (ME alone, isolated, L2 flushed)",
+                             "achieved": me_only_px / 1e12, "peak": peak_px / 1e12, "unit": "Tpx-absdiff/s",
+                             "frac": me_only_px / peak_px},
         "roofline_int": {"bound": "hbm", "kernel": "int_subpel_kernel", "timing": "isolated, L2 flushed",
                          "achieved": u["int_bytes"] * stripe_frac / (int_iso_ms / 1e3) / 1e9,
                          "peak": pk.get("hbm_gbs", 6650.0), "unit": "GB/s",

@@ -17,7 +17,7 @@ import os
 import torch
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libfeves_me.so")
+LIB_PATH = os.environ.get("FEVES_LIB") or os.path.join(_HERE, "libfeves_me.so")   # FEVES_LIB: experiment override
 N_PART = 41
 N_PHASE = 16
 
@@ -58,9 +58,10 @@ def lib():
         L.me_sync.argtypes = [P]
         L.me_set_timing.argtypes = [P, i]
         L.me_get_timings.argtypes = [P, P, P, P]
+        L.me_set_fused.argtypes = [P, i]
         for fn in ("me_set_stream", "me_set_rows", "me_get_layout", "me_estimate", "int_interpolate",
                    "sme_refine", "me_encode_frame", "me_last_launch_count", "me_stream_reset",
-                   "me_stream_push", "me_stream_outputs", "me_sync", "me_set_timing", "me_get_timings"):
+                   "me_stream_push", "me_stream_outputs", "me_sync", "me_set_timing", "me_get_timings", "me_set_fused"):
             getattr(L, fn).restype = i
         _lib = L
     return _lib
@@ -206,6 +207,10 @@ class MotionEstimator:
         _check(lib().me_sync(self._ctx))
 
     # ---------------------------------------------- module timers --
+    def set_fused(self, on: bool = True):
+        """SME fused into the ME kernel (default) or as its own launch."""
+        _check(lib().me_set_fused(self._ctx, int(on)))
+
     def set_timing(self, on: bool = True):
         _check(lib().me_set_timing(self._ctx, int(on)))
 

@@ -47,6 +47,8 @@ struct me_ctx {
   int timing;
   cudaEvent_t ev_t[6];   // INT start/stop (side stream), ME start/stop, SME start/stop
   int timed_mask;        // which pairs were recorded by the last push/encode
+  int fuse;              // run SME inside the ME kernel (me_set_fused)
+  size_t me_smem_fused;
 };
 
 static thread_local int g_last_error = ME_OK;
@@ -75,7 +77,9 @@ static bool is_device_ptr(me_ctx* c, const void* p) {
 
 static cudaError_t set_me_smem(int bytes) {
   cudaError_t e = cudaSuccess;
-  for (auto fn : {me_fsbm_kernel<0>, me_fsbm_kernel<16>, me_fsbm_kernel<32>, me_fsbm_kernel<64>, me_fsbm_kernel<128>})
+  for (auto fn : {me_fsbm_kernel<0>, me_fsbm_kernel<16>, me_fsbm_kernel<32>, me_fsbm_kernel<64>, me_fsbm_kernel<128>,
+                  me_fsbm_kernel<0, true>, me_fsbm_kernel<16, true>, me_fsbm_kernel<32, true>,
+                  me_fsbm_kernel<64, true>, me_fsbm_kernel<128, true>})
     if (e == cudaSuccess) e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
   return e;
 }
@@ -107,6 +111,8 @@ extern "C" me_ctx* me_create(int width, int height, int sa_range, int n_rf) {
   const int S = c->S;
   c->me_threads = me_threads(S);
   c->me_smem = (size_t)me_smem_words(S) * 4;
+  c->me_smem_fused = (size_t)me_smem_words_fused(S, n_rf) * 4;
+  c->fuse = 0;   // measured slower on B200: opt-in
 
   std::vector<uint32_t> rank((size_t)S * S), inv((size_t)(S + 1) * (S + 1), 0);
   for (int dy = -c->R; dy < c->R; ++dy)
@@ -125,7 +131,7 @@ extern "C" me_ctx* me_create(int width, int height, int sa_range, int n_rf) {
     c->own_stream = true;
     ok = cudaMemcpy(c->d_rank, rank.data(), rank.size() * 4, cudaMemcpyHostToDevice) == cudaSuccess &&
          cudaMemcpy(c->d_inv, inv.data(), inv.size() * 4, cudaMemcpyHostToDevice) == cudaSuccess &&
-         set_me_smem((int)c->me_smem) == cudaSuccess;
+         set_me_smem((int)c->me_smem_fused) == cudaSuccess;
   }
   if (!ok) {
     cudaGetLastError();
@@ -202,8 +208,10 @@ static void tmark(me_ctx* c, int i, cudaStream_t st) {
   if (c->timing) { cudaEventRecord(c->ev_t[i], st); c->timed_mask |= 1 << (i / 2); }
 }
 
+// ME (and, when sfs != NULL, the fused SME of me_fsbm.cuh) over n_ref RFs
 static int launch_me(me_ctx* c, const uint8_t* cf, const uint8_t* const* rfs, int16_t* mvs, uint16_t* sads,
-                     int n_ref, cudaStream_t st) {
+                     int n_ref, cudaStream_t st, const uint8_t* const* sfs = nullptr, int16_t* qmvs = nullptr,
+                     uint16_t* qsads = nullptr) {
   MeParams P;
   memset(&P, 0, sizeof(P));
   P.cf = cf;
@@ -215,15 +223,30 @@ static int launch_me(me_ctx* c, const uint8_t* cf, const uint8_t* const* rfs, in
   bool vec = (c->W % 16 == 0) && (c->R % 16 == 0);
   for (int k = 0; k < n_ref; ++k) vec = vec && ((reinterpret_cast<uintptr_t>(rfs[k]) & 15) == 0);
   P.vec_ok = vec ? 1 : 0;
-  dim3 grid(c->mb_cols, c->row1 - c->row0);
-  tmark(c, 2, st);
-  switch (c->S) {   // compile-time window geometry for the paper's SA sizes (Fig. 6a: 32..256)
-    case 16: me_fsbm_kernel<16><<<grid, c->me_threads, c->me_smem, st>>>(P); break;
-    case 32: me_fsbm_kernel<32><<<grid, c->me_threads, c->me_smem, st>>>(P); break;
-    case 64: me_fsbm_kernel<64><<<grid, c->me_threads, c->me_smem, st>>>(P); break;
-    case 128: me_fsbm_kernel<128><<<grid, c->me_threads, c->me_smem, st>>>(P); break;
-    default: me_fsbm_kernel<0><<<grid, c->me_threads, c->me_smem, st>>>(P); break;
+  const bool fused = sfs != nullptr;
+  if (fused) {
+    for (int k = 0; k < n_ref; ++k) P.sf[k] = sfs[k];
+    P.sf_pad = c->sf_pad; P.sf_pitch = c->sf_pitch;
+    P.sf_plane = (size_t)c->sf_rows * c->sf_pitch;
+    P.out_qmvs = reinterpret_cast<uint32_t*>(qmvs);
+    P.out_qsads = qsads;
   }
+  dim3 grid(c->mb_cols, c->row1 - c->row0);
+  const size_t smem = fused ? c->me_smem_fused : c->me_smem;
+  tmark(c, 2, st);
+#define FEVES_ME_LAUNCH(SS)                                                              \
+  do {                                                                                   \
+    if (fused) me_fsbm_kernel<SS, true><<<grid, c->me_threads, smem, st>>>(P);          \
+    else me_fsbm_kernel<SS, false><<<grid, c->me_threads, smem, st>>>(P);               \
+  } while (0)
+  switch (c->S) {   // compile-time window geometry for the paper's SA sizes (Fig. 6a: 32..256)
+    case 16: FEVES_ME_LAUNCH(16); break;
+    case 32: FEVES_ME_LAUNCH(32); break;
+    case 64: FEVES_ME_LAUNCH(64); break;
+    case 128: FEVES_ME_LAUNCH(128); break;
+    default: FEVES_ME_LAUNCH(0); break;
+  }
+#undef FEVES_ME_LAUNCH
   tmark(c, 3, st);
   c->last_launches++;
   return launch_status();
@@ -332,6 +355,9 @@ extern "C" int me_encode_frame(me_ctx* c, const uint8_t* cf, const uint8_t* cons
   int st;
   for (int k = 0; k < n_int; ++k)
     if ((st = launch_int(c, rfs[k], sfs[k], c->stream)) != ME_OK) return st;
+  if (c->fuse)   // ME with the SME fused into the same CTAs (one launch)
+    return launch_me(c, cf, rfs, out_mvs, out_sads, c->n_rf, c->stream, reinterpret_cast<const uint8_t* const*>(sfs),
+                     out_qmvs, out_qsads);
   if ((st = launch_me(c, cf, rfs, mvs, sads, c->n_rf, c->stream)) != ME_OK) return st;
   return launch_sme(c, cf, reinterpret_cast<const uint8_t* const*>(sfs), mvs, sads, out_qmvs, out_qsads, c->n_rf,
                     c->stream);
@@ -387,25 +413,31 @@ extern "C" int me_stream_push(me_ctx* c, const uint8_t* cf, int cf_on_host, int1
   const int n_ref = (int)std::min<long long>(t, c->n_rf);
   if (n_ref_used) *n_ref_used = n_ref;
   if (n_ref > 0) {
-    // side stream: INT of the newest RF (frame t-1), concurrent with ME
     uint8_t* new_rf = c->ring + (size_t)((t - 1) % slots) * fb;
     uint8_t* new_sf = c->sf_ring + (size_t)((t - 1) % c->n_rf) * sb;
-    if (cudaEventRecord(c->ev_fork, c->stream) != cudaSuccess ||
-        cudaStreamWaitEvent(c->side, c->ev_fork, 0) != cudaSuccess)
-      return launch_status();
-    if ((st = launch_int(c, new_rf, new_sf, c->side)) != ME_OK) return st;
-    if (cudaEventRecord(c->ev_join, c->side) != cudaSuccess) return launch_status();
     const uint8_t* rfs[kMaxRf];
     const uint8_t* sfs[kMaxRf];
     for (int k = 0; k < n_ref; ++k) {           // ref_idx k = frame t-1-k
       rfs[k] = c->ring + (size_t)((t - 1 - k) % slots) * fb;
       sfs[k] = c->sf_ring + (size_t)((t - 1 - k) % c->n_rf) * sb;
     }
-    if ((st = launch_me(c, cur, rfs, c->d_mvs, c->d_sads, n_ref, c->stream)) != ME_OK) return st;
-    if (cudaStreamWaitEvent(c->stream, c->ev_join, 0) != cudaSuccess) return launch_status();
     int16_t* qm = (out_qmvs && !out_on_host) ? out_qmvs : c->d_qmvs;
     uint16_t* qs = (out_qsads && !out_on_host) ? out_qsads : c->d_qsads;
-    if ((st = launch_sme(c, cur, sfs, c->d_mvs, c->d_sads, qm, qs, n_ref, c->stream)) != ME_OK) return st;
+    if (c->fuse) {
+      // fused: the SME of ref 0 reads SF(t-1), so INT(t-1) runs first on the same stream
+      if ((st = launch_int(c, new_rf, new_sf, c->stream)) != ME_OK) return st;
+      if ((st = launch_me(c, cur, rfs, nullptr, nullptr, n_ref, c->stream, sfs, qm, qs)) != ME_OK) return st;
+    } else {
+      // side stream: INT of the newest RF (frame t-1), concurrent with ME
+      if (cudaEventRecord(c->ev_fork, c->stream) != cudaSuccess ||
+          cudaStreamWaitEvent(c->side, c->ev_fork, 0) != cudaSuccess)
+        return launch_status();
+      if ((st = launch_int(c, new_rf, new_sf, c->side)) != ME_OK) return st;
+      if (cudaEventRecord(c->ev_join, c->side) != cudaSuccess) return launch_status();
+      if ((st = launch_me(c, cur, rfs, c->d_mvs, c->d_sads, n_ref, c->stream)) != ME_OK) return st;
+      if (cudaStreamWaitEvent(c->stream, c->ev_join, 0) != cudaSuccess) return launch_status();
+      if ((st = launch_sme(c, cur, sfs, c->d_mvs, c->d_sads, qm, qs, n_ref, c->stream)) != ME_OK) return st;
+    }
     const size_t nmv = (size_t)(c->row1 - c->row0) * c->mb_cols * c->n_rf * kNPart;
     if (out_on_host) {
       if ((out_qmvs && cudaMemcpyAsync(out_qmvs, qm, nmv * 4, cudaMemcpyDeviceToHost, c->stream) != cudaSuccess) ||
@@ -449,5 +481,11 @@ extern "C" int me_get_timings(me_ctx* c, float* ms_int, float* ms_me, float* ms_
         cudaEventElapsedTime(out[k], c->ev_t[2 * k], c->ev_t[2 * k + 1]) != cudaSuccess)
       return launch_status();
   }
+  return ME_OK;
+}
+
+extern "C" int me_set_fused(me_ctx* c, int on) {
+  if (!c) return ME_EINVAL;
+  c->fuse = on ? 1 : 0;
   return ME_OK;
 }

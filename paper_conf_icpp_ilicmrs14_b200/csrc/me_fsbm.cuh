@@ -42,6 +42,12 @@ struct MeParams {
   int16_t* out_mvs;
   uint16_t* out_sads;
   int vec_ok;                 // 16-byte aligned rows and window start: vector staging allowed
+  // fused SME (template FUSE): SF of each RF, quarter-pel outputs
+  const uint8_t* sf[kMaxRf];
+  int sf_pad, sf_pitch;
+  size_t sf_plane;
+  uint32_t* out_qmvs;
+  uint16_t* out_qsads;
 };
 
 // ---- launch geometry, shared by host and device (compile-time for the template sizes) ----
@@ -55,6 +61,8 @@ __host__ __device__ constexpr int me_cstride(int S) {                           
 }
 __host__ __device__ constexpr int me_threads(int S) { return 32 * me_ngx(S); }
 __host__ __device__ constexpr int me_smem_words(int S) { return 64 + 4 * me_cstride(S) + (me_threads(S) / 32) * kNPart; }
+// + fused SME: the ME winners of every RF (packed MV, SAD) stay in shared memory
+__host__ __device__ constexpr int me_smem_words_fused(int S, int n_rf) { return me_smem_words(S) + 2 * n_rf * kNPart; }
 
 // Per-candidate aggregation state carried between 4x4 block rows.
 struct RowState {
@@ -155,8 +163,102 @@ __device__ __forceinline__ uint4 lds128_v(const uint32_t* p) {
   return v;
 }
 
-// S_CT = compile-time SA size (0 = any even S read from P at run time)
-template <int S_CT>
+
+// ---------------------------------------------------------------- fused SME --
+// After the ME of its MB, the CTA refines the 41 x n_rf MVs itself (O3; P:86
+// "the MVs from ME define the initial search point for the SME"): 16 lanes per
+// RF, lane = one 4x4 block (bits bx0, by0, bx1, by1 so every partition of every
+// mode is an xor-closed lane set), CF from shared memory, SF from L2/HBM.  The
+// SME phase is memory-latency-bound and the ME phase ALU-bound, so while one CTA
+// refines, the other resident CTAs of the SM keep the ALU pipe busy.
+// ring-1 spiral order s_k (G12/G14): (0,-1),(0,1),(-1,-1),(1,-1),(-1,0),(1,0),(-1,1),(1,1)
+__host__ __device__ constexpr int ring_x(int k) { return k < 2 ? 0 : ((k & 1) ? 1 : -1); }
+__host__ __device__ constexpr int ring_y(int k) { return k < 2 ? ((k & 1) ? 1 : -1) : (k < 4 ? -1 : k < 6 ? 0 : 1); }
+
+__device__ __forceinline__ uint32_t fsme_block_sad(const uint8_t* __restrict__ sf, size_t plane, int pitch, int pad,
+                                                   int bxp, int byp, int vx, int vy, const uint32_t (&cfb)[4]) {
+  const uint8_t* pl = sf + (size_t)(4 * (vy & 3) + (vx & 3)) * plane;
+  const uint8_t* p0 = pl + (size_t)(byp + (vy >> 2) + pad) * pitch + (bxp + (vx >> 2) + pad);
+  const uintptr_t a = reinterpret_cast<uintptr_t>(p0);
+  const uint32_t* w = reinterpret_cast<const uint32_t*>(a & ~uintptr_t(3));
+  const uint32_t sh = 8u * (uint32_t)(a & 3);
+  const int wp = pitch >> 2;
+  uint32_t s = 0;
+#pragma unroll
+  for (int r = 0; r < 4; ++r) {
+    const uint32_t lo = __ldg(w + r * wp), hi = __ldg(w + r * wp + 1);
+    s = vad4(cfb[r], __funnelshift_r(lo, hi, sh), s);
+  }
+  return s;
+}
+
+template <int MASK>
+__device__ __forceinline__ uint32_t fsme_sum(uint32_t v) {   // all-reduce inside the 16-lane half
+  const unsigned half = (threadIdx.x & 16) ? 0xffff0000u : 0x0000ffffu;
+  if (MASK & 1) v += __shfl_xor_sync(half, v, 1);
+  if (MASK & 2) v += __shfl_xor_sync(half, v, 2);
+  if (MASK & 4) v += __shfl_xor_sync(half, v, 4);
+  if (MASK & 8) v += __shfl_xor_sync(half, v, 8);
+  return v;
+}
+
+template <int MASK>
+__device__ __forceinline__ void fsme_mode(const MeParams& P, const uint8_t* __restrict__ sf, int p, size_t o,
+                                          const uint32_t* mvs_s, const uint32_t* sads_s, int bxp, int byp, int b,
+                                          const uint32_t (&cfb)[4]) {
+  const uint32_t mv = mvs_s[p];
+  const int cx = 4 * (int)(int16_t)(mv & 0xffffu), cy = 4 * (int)(int16_t)(mv >> 16);
+  uint32_t best = sads_s[p];                  // centre cost = the ME SAD (phase 0 = integer samples)
+  int bvx = cx, bvy = cy;
+#pragma unroll
+  for (int stage = 0; stage < 2; ++stage) {
+    const int ox = bvx, oy = bvy;             // half: around c; quarter: around the best half position
+    uint32_t sad[8];
+#pragma unroll
+    for (int k = 0; k < 8; ++k)
+      sad[k] = fsme_block_sad(sf, P.sf_plane, P.sf_pitch, P.sf_pad, bxp, byp, ox + (ring_x(k) << (1 - stage)),
+                              oy + (ring_y(k) << (1 - stage)), cfb);
+#pragma unroll
+    for (int k = 0; k < 8; ++k) {             // spiral order, strict < (G14)
+      const uint32_t t = fsme_sum<MASK>(sad[k]);
+      if (t < best) { best = t; bvx = ox + (ring_x(k) << (1 - stage)); bvy = oy + (ring_y(k) << (1 - stage)); }
+    }
+  }
+  if ((b & MASK) == 0) {                      // partition leader writes
+    P.out_qmvs[o + p] = (uint32_t)(uint16_t)bvx | ((uint32_t)(uint16_t)bvy << 16);
+    P.out_qsads[o + p] = (uint16_t)best;
+  }
+}
+
+__device__ __forceinline__ void fused_sme(const MeParams& P, const uint32_t* cf_s, const uint32_t* win_mv,
+                                          const uint32_t* win_sad, int mbx) {
+  const int b = threadIdx.x & 15;
+  const int bx0 = b & 1, by0 = (b >> 1) & 1, bx1 = (b >> 2) & 1, by1 = (b >> 3) & 1;
+  const int bx = 2 * bx1 + bx0, by = 2 * by1 + by0;
+  const int bxp = 16 * mbx + 4 * bx, byp = 16 * (P.row0 + blockIdx.y) + 4 * by;
+  uint32_t cfb[4];
+#pragma unroll
+  for (int r = 0; r < 4; ++r) cfb[r] = cf_s[(4 * by + r) * 4 + bx];
+  const int s = 2 * by1 + bx1;
+  const int groups = blockDim.x >> 4;
+  for (int ref = threadIdx.x >> 4; ref < P.n_rf; ref += groups) {   // whole 16-lane halves iterate together
+    const uint8_t* __restrict__ sf = P.sf[ref];
+    const uint32_t* mvs_s = win_mv + ref * kNPart;
+    const uint32_t* sads_s = win_sad + ref * kNPart;
+    const size_t o = ((size_t)(blockIdx.y * P.mb_cols + mbx) * P.rf_stride + ref) * kNPart;
+    fsme_mode<15>(P, sf, 0, o, mvs_s, sads_s, bxp, byp, b, cfb);                           // 16x16
+    fsme_mode<7>(P, sf, 1 + by1, o, mvs_s, sads_s, bxp, byp, b, cfb);                      // 16x8
+    fsme_mode<11>(P, sf, 3 + bx1, o, mvs_s, sads_s, bxp, byp, b, cfb);                     // 8x16
+    fsme_mode<3>(P, sf, 5 + s, o, mvs_s, sads_s, bxp, byp, b, cfb);                        // 8x8
+    fsme_mode<1>(P, sf, 9 + 2 * s + by0, o, mvs_s, sads_s, bxp, byp, b, cfb);              // 8x4
+    fsme_mode<2>(P, sf, 17 + 2 * s + bx0, o, mvs_s, sads_s, bxp, byp, b, cfb);             // 4x8
+    fsme_mode<0>(P, sf, 25 + 4 * s + 2 * by0 + bx0, o, mvs_s, sads_s, bxp, byp, b, cfb);   // 4x4
+  }
+}
+
+// S_CT = compile-time SA size (0 = any even S read from P at run time);
+// FUSE = also run the SME of this MB (fused_sme) after its ME.
+template <int S_CT, bool FUSE = false>
 __global__ void __launch_bounds__(128, 4) me_fsbm_kernel(const MeParams P) {
   extern __shared__ __align__(16) uint32_t smem[];
   const int S = S_CT ? S_CT : P.S;
@@ -166,6 +268,8 @@ __global__ void __launch_bounds__(128, 4) me_fsbm_kernel(const MeParams P) {
   uint32_t* cf_s = smem;                                  // 16 rows x 4 words
   uint32_t* win = smem + 64;                              // 4 copies x CSTRIDE words
   uint32_t* red = win + 4 * CSTRIDE;                      // [nwarps][41]
+  uint32_t* win_mv = red + (blockDim.x >> 5) * kNPart;    // FUSE: [n_rf][41] packed MVs, then SADs
+  uint32_t* win_sad = win_mv + P.n_rf * kNPart;
 
   const int mbx = blockIdx.x, mby = P.row0 + blockIdx.y;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -294,9 +398,19 @@ __global__ void __launch_bounds__(128, 4) me_fsbm_kernel(const MeParams P) {
       for (int w = 1; w < nwarps; ++w) k = min(k, red[w * kNPart + p]);
       const uint32_t mv = __ldg(P.inv_tab + (k & 0xffffu));
       const size_t o = ((size_t)(blockIdx.y * P.mb_cols + mbx) * P.rf_stride + ref) * kNPart + p;
-      reinterpret_cast<uint32_t*>(P.out_mvs)[o] = mv;
-      P.out_sads[o] = (uint16_t)(k >> 16);
+      if (P.out_mvs) {
+        reinterpret_cast<uint32_t*>(P.out_mvs)[o] = mv;
+        P.out_sads[o] = (uint16_t)(k >> 16);
+      }
+      if (FUSE) {
+        win_mv[ref * kNPart + p] = mv;
+        win_sad[ref * kNPart + p] = k >> 16;
+      }
     }
+  }
+  if (FUSE) {
+    __syncthreads();
+    fused_sme(P, cf_s, win_mv, win_sad, mbx);
   }
 }
 

@@ -133,12 +133,36 @@ def test_encode_frame_equals_separate_calls(feves):
     mvs, sads = me.estimate(tcf, trfs)
     qa, sa = me.refine(tcf, sfs_a, mvs, sads)
     sfs_b = [me.new_sf() for _ in trfs]
+    me.set_fused(True)
     (m2, s2), (qb, sb) = me.encode_frame(tcf, trfs, sfs_b, n_int=2, out_me=me.new_mvs())
-    assert me.launches == 2 * 2 + 2          # INT interior + border launch per RF, ME, SME
+    assert me.launches == 2 * 2 + 1          # INT interior + border launch per RF, fused ME+SME
+    me.set_fused(False)
+    sfs_c = [me.new_sf() for _ in trfs]
+    (m3, s3), (qc, sc) = me.encode_frame(tcf, trfs, sfs_c, n_int=2, out_me=me.new_mvs())
+    assert me.launches == 2 * 2 + 2          # ... ME, SME as separate launches
     torch.cuda.synchronize()
     assert torch.equal(mvs, m2) and torch.equal(sads, s2) and torch.equal(qa, qb) and torch.equal(sa, sb)
-    for a, b in zip(sfs_a, sfs_b):
-        assert torch.equal(a, b)
+    assert torch.equal(mvs, m3) and torch.equal(sads, s3) and torch.equal(qa, qc) and torch.equal(sa, sc)
+    for a, b, c in zip(sfs_a, sfs_b, sfs_c):
+        assert torch.equal(a, b) and torch.equal(a, c)
+    me.close()
+
+
+@pytest.mark.parametrize("fused", [True, False])
+def test_stream_fused_and_unfused_agree(feves, orc, fused):
+    W, H, S, n_rf = 96, 64, 32, 2
+    frames = [gen_noise(W, H, t, 17) for t in range(4)]
+    me = feves.MotionEstimator(W, H, S, n_rf)
+    me.set_fused(fused)
+    for f in frames:
+        qm, qs, used = me.stream_push(_dev(f))
+    torch.cuda.synchronize()
+    n = me.mb_rows * me.mb_cols
+    rfs = [frames[2], frames[1]]
+    o_mvs, _ = orc.me(frames[3], rfs, S)
+    o_q, o_s = orc.sme(frames[3], rfs, o_mvs)
+    np.testing.assert_array_equal(qm.cpu().numpy().reshape(n, n_rf, 41, 2), o_q)
+    np.testing.assert_array_equal(qs.cpu().numpy().reshape(n, n_rf, 41), o_s)
     me.close()
 
 
