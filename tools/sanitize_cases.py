@@ -1,0 +1,25 @@
+"""Small ME/INT/SME/stream cases for compute-sanitizer (no oracle, no asserts: the tool checks)."""
+import sys, os
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import numpy as np
+import torch
+import paper_conf_icpp_ilicmrs14_b200 as F
+from synth import gen_tex
+
+for (W, H, S, n) in [(64, 48, 16, 2), (37, 29, 8, 1), (96, 80, 64, 2), (48, 40, 128, 1)]:
+    frames = [torch.from_numpy(gen_tex(W, H, t, 1)).cuda() for t in range(n + 2)]
+    me = F.MotionEstimator(W, H, S, n)
+    sfs = [me.new_sf() for _ in range(n)]
+    me.encode_frame(frames[n], frames[:n], sfs, n_int=n, out_me=me.new_mvs())
+    me.set_fused(True)
+    me.encode_frame(frames[n], frames[:n], sfs, n_int=n, out_me=me.new_mvs())
+    me.set_fused(False)
+    for f in frames:
+        me.stream_push(f)
+    me.set_rows(0, 1)
+    me.stream_reset()
+    for f in frames:
+        me.stream_push(f)
+    torch.cuda.synchronize()
+    me.close()
+print("sanitize cases done")
