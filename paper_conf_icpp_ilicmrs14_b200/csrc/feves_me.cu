@@ -43,6 +43,14 @@ struct me_ctx {
   long long t;           // frames pushed since reset
   cudaStream_t side;     // INT runs here, concurrently with ME
   cudaEvent_t ev_fork, ev_join;
+  // host-buffer pushes: uploads / downloads on their own streams so the copy engines
+  // overlap the compute of the neighbouring frames (P:51 copy engines, Fig. 4 VCM)
+  cudaStream_t copy_in, copy_out;
+  cudaEvent_t ev_done[2];     // compute of push t finished (ring: t & 1)
+  cudaEvent_t ev_up[2];       // upload of push t finished
+  cudaEvent_t ev_down[2];     // download of push t finished (frees device output buffer t & 1)
+  int16_t* d_qmvs2[2];        // double-buffered device outputs for host pushes
+  uint16_t* d_qsads2[2];
   // per-module timers ("facilities to measure execution ... times")
   int timing;
   cudaEvent_t ev_t[6];   // INT start/stop (side stream), ME start/stop, SME start/stop
@@ -145,7 +153,10 @@ extern "C" me_ctx* me_create(int width, int height, int sa_range, int n_rf) {
 
 extern "C" void me_destroy(me_ctx* c) {
   if (!c) return;
-  if (c->own_stream && c->stream) cudaStreamSynchronize(c->stream);
+  if (c->stream) cudaStreamSynchronize(c->stream);
+  if (c->copy_in) cudaStreamSynchronize(c->copy_in);
+  if (c->copy_out) cudaStreamSynchronize(c->copy_out);
+  if (c->side) cudaStreamSynchronize(c->side);
   cudaFree(c->d_rank);
   cudaFree(c->d_inv);
   cudaFree(c->d_mvs);
@@ -156,6 +167,15 @@ extern "C" void me_destroy(me_ctx* c) {
   cudaFree(c->d_qsads);
   for (int i = 0; i < 6; ++i)
     if (c->ev_t[i]) cudaEventDestroy(c->ev_t[i]);
+  for (int i = 0; i < 2; ++i) {
+    if (c->ev_done[i]) cudaEventDestroy(c->ev_done[i]);
+    if (c->ev_up[i]) cudaEventDestroy(c->ev_up[i]);
+    if (c->ev_down[i]) cudaEventDestroy(c->ev_down[i]);
+    cudaFree(c->d_qmvs2[i]);
+    cudaFree(c->d_qsads2[i]);
+  }
+  if (c->copy_in) cudaStreamDestroy(c->copy_in);
+  if (c->copy_out) cudaStreamDestroy(c->copy_out);
   if (c->side) cudaStreamDestroy(c->side);
   if (c->ev_fork) cudaEventDestroy(c->ev_fork);
   if (c->ev_join) cudaEventDestroy(c->ev_join);
@@ -377,16 +397,30 @@ extern "C" int me_stream_reset(me_ctx* c) {
   return ME_OK;
 }
 
+// ring of n_rf + 2 frames: the slot written by push t held frame t-n_rf-2, last
+// read by the compute of push t-2, so the upload of t overlaps the compute of t-1
+static int ring_slots(const me_ctx* c) { return c->n_rf + 2; }
+
 static int stream_alloc(me_ctx* c) {
   if (c->ring) return ME_OK;
   const size_t fb = (size_t)c->W * c->H, sb = (size_t)kNPhase * c->sf_rows * c->sf_pitch;
   const size_t nmv = (size_t)c->mb_cols * c->mb_rows * c->n_rf * kNPart;
-  if (cudaMalloc(&c->ring, fb * (c->n_rf + 1)) != cudaSuccess ||
-      cudaMalloc(&c->sf_ring, sb * c->n_rf) != cudaSuccess || cudaMalloc(&c->d_qmvs, nmv * 4) != cudaSuccess ||
-      cudaMalloc(&c->d_qsads, nmv * 2) != cudaSuccess ||
-      cudaStreamCreateWithFlags(&c->side, cudaStreamNonBlocking) != cudaSuccess ||
-      cudaEventCreateWithFlags(&c->ev_fork, cudaEventDisableTiming) != cudaSuccess ||
-      cudaEventCreateWithFlags(&c->ev_join, cudaEventDisableTiming) != cudaSuccess) {
+  bool ok = cudaMalloc(&c->ring, fb * ring_slots(c)) == cudaSuccess &&
+            cudaMalloc(&c->sf_ring, sb * c->n_rf) == cudaSuccess && cudaMalloc(&c->d_qmvs, nmv * 4) == cudaSuccess &&
+            cudaMalloc(&c->d_qsads, nmv * 2) == cudaSuccess &&
+            cudaStreamCreateWithFlags(&c->side, cudaStreamNonBlocking) == cudaSuccess &&
+            cudaStreamCreateWithFlags(&c->copy_in, cudaStreamNonBlocking) == cudaSuccess &&
+            cudaStreamCreateWithFlags(&c->copy_out, cudaStreamNonBlocking) == cudaSuccess &&
+            cudaEventCreateWithFlags(&c->ev_fork, cudaEventDisableTiming) == cudaSuccess &&
+            cudaEventCreateWithFlags(&c->ev_join, cudaEventDisableTiming) == cudaSuccess;
+  for (int i = 0; ok && i < 2; ++i)
+    ok = cudaEventCreateWithFlags(&c->ev_done[i], cudaEventDisableTiming) == cudaSuccess &&
+         cudaEventCreateWithFlags(&c->ev_up[i], cudaEventDisableTiming) == cudaSuccess &&
+         cudaEventCreateWithFlags(&c->ev_down[i], cudaEventDisableTiming) == cudaSuccess &&
+         cudaMalloc(&c->d_qmvs2[i], nmv * 4) == cudaSuccess && cudaMalloc(&c->d_qsads2[i], nmv * 2) == cudaSuccess &&
+         cudaEventRecord(c->ev_done[i], c->stream) == cudaSuccess &&     // "already done" for t < 2
+         cudaEventRecord(c->ev_down[i], c->stream) == cudaSuccess;
+  if (!ok) {
     cudaGetLastError();
     return ME_ENOMEM;
   }
@@ -404,12 +438,20 @@ extern "C" int me_stream_push(me_ctx* c, const uint8_t* cf, int cf_on_host, int1
   c->last_launches = 0;
   c->timed_mask = 0;
   const size_t fb = (size_t)c->W * c->H, sb = (size_t)kNPhase * c->sf_rows * c->sf_pitch;
-  const int slots = c->n_rf + 1;
+  const int slots = ring_slots(c);
   const long long t = c->t;
+  const int par = (int)(t & 1);
   uint8_t* cur = c->ring + (size_t)(t % slots) * fb;
-  if (cudaMemcpyAsync(cur, cf, fb, cf_on_host ? cudaMemcpyHostToDevice : cudaMemcpyDeviceToDevice, c->stream) !=
-      cudaSuccess)
+  if (cf_on_host) {
+    // upload on the copy-in stream once the compute of push t-2 (last reader of this slot) is done
+    if (cudaStreamWaitEvent(c->copy_in, c->ev_done[par], 0) != cudaSuccess ||
+        cudaMemcpyAsync(cur, cf, fb, cudaMemcpyHostToDevice, c->copy_in) != cudaSuccess ||
+        cudaEventRecord(c->ev_up[par], c->copy_in) != cudaSuccess ||
+        cudaStreamWaitEvent(c->stream, c->ev_up[par], 0) != cudaSuccess)
+      return launch_status();
+  } else if (cudaMemcpyAsync(cur, cf, fb, cudaMemcpyDeviceToDevice, c->stream) != cudaSuccess) {
     return launch_status();
+  }
   const int n_ref = (int)std::min<long long>(t, c->n_rf);
   if (n_ref_used) *n_ref_used = n_ref;
   if (n_ref > 0) {
@@ -421,8 +463,10 @@ extern "C" int me_stream_push(me_ctx* c, const uint8_t* cf, int cf_on_host, int1
       rfs[k] = c->ring + (size_t)((t - 1 - k) % slots) * fb;
       sfs[k] = c->sf_ring + (size_t)((t - 1 - k) % c->n_rf) * sb;
     }
-    int16_t* qm = (out_qmvs && !out_on_host) ? out_qmvs : c->d_qmvs;
-    uint16_t* qs = (out_qsads && !out_on_host) ? out_qsads : c->d_qsads;
+    int16_t* qm = (out_qmvs && !out_on_host) ? out_qmvs : (out_on_host ? c->d_qmvs2[par] : c->d_qmvs);
+    uint16_t* qs = (out_qsads && !out_on_host) ? out_qsads : (out_on_host ? c->d_qsads2[par] : c->d_qsads);
+    // the device output buffer t & 1 is free once the download of push t-2 finished
+    if (out_on_host && cudaStreamWaitEvent(c->stream, c->ev_down[par], 0) != cudaSuccess) return launch_status();
     if (c->fuse) {
       // fused: the SME of ref 0 reads SF(t-1), so INT(t-1) runs first on the same stream
       if ((st = launch_int(c, new_rf, new_sf, c->stream)) != ME_OK) return st;
@@ -439,11 +483,16 @@ extern "C" int me_stream_push(me_ctx* c, const uint8_t* cf, int cf_on_host, int1
       if ((st = launch_sme(c, cur, sfs, c->d_mvs, c->d_sads, qm, qs, n_ref, c->stream)) != ME_OK) return st;
     }
     const size_t nmv = (size_t)(c->row1 - c->row0) * c->mb_cols * c->n_rf * kNPart;
-    if (out_on_host) {
-      if ((out_qmvs && cudaMemcpyAsync(out_qmvs, qm, nmv * 4, cudaMemcpyDeviceToHost, c->stream) != cudaSuccess) ||
-          (out_qsads && cudaMemcpyAsync(out_qsads, qs, nmv * 2, cudaMemcpyDeviceToHost, c->stream) != cudaSuccess))
+    if (cudaEventRecord(c->ev_done[par], c->stream) != cudaSuccess) return launch_status();
+    if (out_on_host) {   // download on the copy-out stream, overlapping the next frame's compute
+      if (cudaStreamWaitEvent(c->copy_out, c->ev_done[par], 0) != cudaSuccess ||
+          (out_qmvs && cudaMemcpyAsync(out_qmvs, qm, nmv * 4, cudaMemcpyDeviceToHost, c->copy_out) != cudaSuccess) ||
+          (out_qsads && cudaMemcpyAsync(out_qsads, qs, nmv * 2, cudaMemcpyDeviceToHost, c->copy_out) != cudaSuccess) ||
+          cudaEventRecord(c->ev_down[par], c->copy_out) != cudaSuccess)
         return launch_status();
     }
+  } else if (cudaEventRecord(c->ev_done[par], c->stream) != cudaSuccess) {
+    return launch_status();
   }
   c->t = t + 1;
   return ME_OK;
@@ -451,7 +500,11 @@ extern "C" int me_stream_push(me_ctx* c, const uint8_t* cf, int cf_on_host, int1
 
 extern "C" int me_sync(me_ctx* c) {
   if (!c) return ME_EINVAL;
-  return cudaStreamSynchronize(c->stream) == cudaSuccess ? ME_OK : ME_ECUDA;
+  cudaError_t e = cudaStreamSynchronize(c->stream);
+  if (e == cudaSuccess && c->copy_in) e = cudaStreamSynchronize(c->copy_in);
+  if (e == cudaSuccess && c->copy_out) e = cudaStreamSynchronize(c->copy_out);
+  if (e == cudaSuccess && c->side) e = cudaStreamSynchronize(c->side);
+  return e == cudaSuccess ? ME_OK : ME_ECUDA;
 }
 
 extern "C" int me_stream_outputs(me_ctx* c, int16_t** qmvs, uint16_t** qsads) {

@@ -300,3 +300,26 @@ def test_stream_push_host_buffers(feves, orc):
     np.testing.assert_array_equal(qm.numpy().reshape(n, n_rf, 41, 2), o_q)
     np.testing.assert_array_equal(qs.numpy().reshape(n, n_rf, 41), o_s)
     me.close()
+
+
+def test_stream_host_pipeline_many_frames(feves, orc):
+    """host pushes back to back (uploads/downloads overlap compute on copy streams):
+    every frame's host outputs, captured into its own pinned buffer, match the oracle"""
+    W, H, S, n_rf = 64, 48, 8, 2
+    frames = [gen_tex(W, H, t, 23) for t in range(7)]
+    me = feves.MotionEstimator(W, H, S, n_rf)
+    n = me.mb_rows * me.mb_cols
+    outs = []
+    for f in frames:
+        o = (torch.empty(me.mv_shape() + (2,), dtype=torch.int16).pin_memory(),
+             torch.empty(me.mv_shape(), dtype=torch.uint16).pin_memory())
+        me.stream_push(torch.from_numpy(f).pin_memory(), out=o)
+        outs.append(o)
+    me.sync()
+    for t in range(n_rf, len(frames)):
+        rfs = [frames[t - 1 - k] for k in range(n_rf)]
+        o_mvs, _ = orc.me(frames[t], rfs, S)
+        o_q, o_s = orc.sme(frames[t], rfs, o_mvs)
+        np.testing.assert_array_equal(outs[t][0].numpy().reshape(n, n_rf, 41, 2), o_q)
+        np.testing.assert_array_equal(outs[t][1].numpy().reshape(n, n_rf, 41), o_s)
+    me.close()
