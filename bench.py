@@ -48,6 +48,9 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-budget", type=float, default=10.0, help="seconds of oracle wall time")
+    ap.add_argument("--pipeline", type=int, default=None, help="ME_OPT_PIPELINE_RF (default: library default)")
+    ap.add_argument("--me-ctas", type=int, default=None, help="ME_OPT_ME_CTAS_PER_SM")
+    ap.add_argument("--fused", type=int, default=None, help="ME_OPT_FUSED_SME")
     return ap.parse_args()
 
 
@@ -222,6 +225,10 @@ def run_feves(args, cfg):
     me = feves.MotionEstimator(cfg.width, cfg.height, cfg.sa_range, cfg.n_rf, device=dev)
     r0, r1 = stripes(me.mb_rows, world)[rank]
     me.set_rows(r0, r1)
+    for opt, val in ((me.OPT_PIPELINE_RF, args.pipeline), (me.OPT_ME_CTAS_PER_SM, args.me_ctas),
+                     (me.OPT_FUSED_SME, args.fused)):
+        if val is not None:
+            me.set_option(opt, val)
     me.set_timing(True)
     stream = torch.cuda.current_stream(dev)
 
@@ -317,6 +324,34 @@ def run_feves(args, cfg):
 
     # ---- e2e: pinned host frame in, host MVs/SADs out, every step ----
     e2e = None
+    if not args.no_e2e and world > 1:
+        # sharded: rank 0 uploads the pinned frame, broadcast + per-rank push + gather
+        # (ShardedStream), rank 0 downloads the assembled quarter-pel MVs + SADs
+        me.stream_reset()
+        for i in range(cfg.n_rf + 2):
+            ss.push(frames[i % n_frames], buf)
+        torch.cuda.synchronize()
+        dist.barrier()
+        qm_h = torch.empty((me.mb_rows, me.mb_cols, cfg.n_rf, 41, 2), dtype=torch.int16).pin_memory()
+        qs_h = torch.empty((me.mb_rows, me.mb_cols, cfg.n_rf, 41), dtype=torch.uint16).pin_memory()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        for i in range(args.e2e_steps):
+            if rank == 0:
+                buf.copy_(pinned[(cfg.n_rf + 2 + i) % n_frames], non_blocking=True)
+            r = ss.push(buf, buf)
+            if rank == 0:
+                qm_h.copy_(r[0], non_blocking=True)
+                qs_h.copy_(r[1], non_blocking=True)
+        e1.record(stream)
+        torch.cuda.synchronize()
+        tt = torch.tensor([e0.elapsed_time(e1)], dtype=torch.float64, device=dev)
+        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+        e2e = {"value": args.e2e_steps / (float(tt.item()) / 1e3), "unit": "frames/s",
+               "h2d_bytes_per_step": pinned[0].numel(),
+               "d2h_bytes_per_step": qm_h.numel() * 2 + qs_h.numel() * 2,
+               "api": "ShardedStream.push (NCCL broadcast in, per-rank me_stream_push, NCCL gather out), "
+                      "pinned buffers on rank 0"}
     if not args.no_e2e and world == 1:
         qm_h = torch.empty(me.mv_shape() + (2,), dtype=torch.int16).pin_memory()
         qs_h = torch.empty(me.mv_shape(), dtype=torch.uint16).pin_memory()

@@ -59,9 +59,10 @@ def lib():
         L.me_set_timing.argtypes = [P, i]
         L.me_get_timings.argtypes = [P, P, P, P]
         L.me_set_fused.argtypes = [P, i]
+        L.me_set_option.argtypes = [P, i, i]
         for fn in ("me_set_stream", "me_set_rows", "me_get_layout", "me_estimate", "int_interpolate",
                    "sme_refine", "me_encode_frame", "me_last_launch_count", "me_stream_reset",
-                   "me_stream_push", "me_stream_outputs", "me_sync", "me_set_timing", "me_get_timings", "me_set_fused"):
+                   "me_stream_push", "me_stream_outputs", "me_sync", "me_set_timing", "me_get_timings", "me_set_fused", "me_set_option"):
             getattr(L, fn).restype = i
         _lib = L
     return _lib
@@ -210,6 +211,12 @@ class MotionEstimator:
     def set_fused(self, on: bool = True):
         """SME fused into the ME kernel (default) or as its own launch."""
         _check(lib().me_set_fused(self._ctx, int(on)))
+
+    OPT_FUSED_SME, OPT_PIPELINE_RF, OPT_ME_CTAS_PER_SM = 1, 2, 3
+
+    def set_option(self, option: int, value: int):
+        """me_set_option: scheduling knobs (results identical under every setting)."""
+        _check(lib().me_set_option(self._ctx, option, value))
 
     def set_timing(self, on: bool = True):
         _check(lib().me_set_timing(self._ctx, int(on)))

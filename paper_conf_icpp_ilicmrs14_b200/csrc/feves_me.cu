@@ -55,8 +55,12 @@ struct me_ctx {
   int timing;
   cudaEvent_t ev_t[6];   // INT start/stop (side stream), ME start/stop, SME start/stop
   int timed_mask;        // which pairs were recorded by the last push/encode
-  int fuse;              // run SME inside the ME kernel (me_set_fused)
+  int fuse;              // run SME inside the ME kernel (ME_OPT_FUSED_SME)
   size_t me_smem_fused;
+  int pipeline;          // per-RF ME launches, SME of RF k co-running with ME of RF k+1 (ME_OPT_PIPELINE_RF)
+  int me_ctas_per_sm;    // cap on resident ME CTAs per SM (0 = hardware maximum; ME_OPT_ME_CTAS_PER_SM)
+  cudaStream_t sme_st;   // pipeline: SME stream
+  cudaEvent_t ev_me[kMaxRf], ev_sme_done;
 };
 
 static thread_local int g_last_error = ME_OK;
@@ -121,6 +125,8 @@ extern "C" me_ctx* me_create(int width, int height, int sa_range, int n_rf) {
   c->me_smem = (size_t)me_smem_words(S) * 4;
   c->me_smem_fused = (size_t)me_smem_words_fused(S, n_rf) * 4;
   c->fuse = 0;   // measured slower on B200: opt-in
+  c->pipeline = 0;
+  c->me_ctas_per_sm = 0;
 
   std::vector<uint32_t> rank((size_t)S * S), inv((size_t)(S + 1) * (S + 1), 0);
   for (int dy = -c->R; dy < c->R; ++dy)
@@ -139,7 +145,7 @@ extern "C" me_ctx* me_create(int width, int height, int sa_range, int n_rf) {
     c->own_stream = true;
     ok = cudaMemcpy(c->d_rank, rank.data(), rank.size() * 4, cudaMemcpyHostToDevice) == cudaSuccess &&
          cudaMemcpy(c->d_inv, inv.data(), inv.size() * 4, cudaMemcpyHostToDevice) == cudaSuccess &&
-         set_me_smem((int)c->me_smem_fused) == cudaSuccess;
+         set_me_smem(200 * 1024) == cudaSuccess;   // max; the launch asks for what it needs
   }
   if (!ok) {
     cudaGetLastError();
@@ -157,6 +163,7 @@ extern "C" void me_destroy(me_ctx* c) {
   if (c->copy_in) cudaStreamSynchronize(c->copy_in);
   if (c->copy_out) cudaStreamSynchronize(c->copy_out);
   if (c->side) cudaStreamSynchronize(c->side);
+  if (c->sme_st) cudaStreamSynchronize(c->sme_st);
   cudaFree(c->d_rank);
   cudaFree(c->d_inv);
   cudaFree(c->d_mvs);
@@ -174,6 +181,10 @@ extern "C" void me_destroy(me_ctx* c) {
     cudaFree(c->d_qmvs2[i]);
     cudaFree(c->d_qsads2[i]);
   }
+  for (int i = 0; i < kMaxRf; ++i)
+    if (c->ev_me[i]) cudaEventDestroy(c->ev_me[i]);
+  if (c->ev_sme_done) cudaEventDestroy(c->ev_sme_done);
+  if (c->sme_st) cudaStreamDestroy(c->sme_st);
   if (c->copy_in) cudaStreamDestroy(c->copy_in);
   if (c->copy_out) cudaStreamDestroy(c->copy_out);
   if (c->side) cudaStreamDestroy(c->side);
@@ -252,7 +263,9 @@ static int launch_me(me_ctx* c, const uint8_t* cf, const uint8_t* const* rfs, in
     P.out_qsads = qsads;
   }
   dim3 grid(c->mb_cols, c->row1 - c->row0);
-  const size_t smem = fused ? c->me_smem_fused : c->me_smem;
+  size_t smem = fused ? c->me_smem_fused : c->me_smem;
+  if (c->me_ctas_per_sm > 0)   // occupancy cap: leave registers / warps for a co-running SME
+    smem = std::max(smem, (size_t)(228 * 1024) / (size_t)(c->me_ctas_per_sm + 1) - 1024 + 64);
   tmark(c, 2, st);
 #define FEVES_ME_LAUNCH(SS)                                                              \
   do {                                                                                   \
@@ -330,6 +343,48 @@ static int launch_sme(me_ctx* c, const uint8_t* cf, const uint8_t* const* sfs, c
   return launch_status();
 }
 
+// ME then SME of n_ref RFs.  Pipelined (ME_OPT_PIPELINE_RF): one ME launch per RF on
+// the compute stream, and the SME of RF k on the SME stream as soon as the ME of RF k
+// is done (the only dependency), so the memory-latency-bound SME of RF k co-runs
+// with the ALU-bound ME of RF k+1.  sf_ready (may be null) gates the first SME.
+static int run_me_sme(me_ctx* c, const uint8_t* cf, const uint8_t* const* rfs, const uint8_t* const* sfs,
+                      int16_t* mvs, uint16_t* sads, int16_t* qmvs, uint16_t* qsads, int n_ref, cudaEvent_t sf_ready) {
+  int st;
+  if (!c->pipeline) {
+    if ((st = launch_me(c, cf, rfs, mvs, sads, n_ref, c->stream)) != ME_OK) return st;
+    if (sf_ready && cudaStreamWaitEvent(c->stream, sf_ready, 0) != cudaSuccess) return launch_status();
+    return launch_sme(c, cf, sfs, mvs, sads, qmvs, qsads, n_ref, c->stream);
+  }
+  if (!c->sme_st) {
+    if (cudaStreamCreateWithFlags(&c->sme_st, cudaStreamNonBlocking) != cudaSuccess ||
+        cudaEventCreateWithFlags(&c->ev_sme_done, cudaEventDisableTiming) != cudaSuccess)
+      return launch_status();
+    for (int k = 0; k < kMaxRf; ++k)
+      if (cudaEventCreateWithFlags(&c->ev_me[k], cudaEventDisableTiming) != cudaSuccess) return launch_status();
+  }
+  const int saved = c->timing;
+  c->timing = 0;   // per-module timers are not meaningful for interleaved launches
+  // the SME stream must see everything enqueued on the compute stream so far
+  if (cudaEventRecord(c->ev_sme_done, c->stream) != cudaSuccess ||
+      cudaStreamWaitEvent(c->sme_st, c->ev_sme_done, 0) != cudaSuccess)
+    return launch_status();
+  if (sf_ready && cudaStreamWaitEvent(c->sme_st, sf_ready, 0) != cudaSuccess) return launch_status();
+  for (int k = 0; k < n_ref; ++k) {
+    const size_t off = (size_t)k * kNPart;
+    if ((st = launch_me(c, cf, rfs + k, mvs + 2 * off, sads + off, 1, c->stream)) != ME_OK) return st;
+    if (cudaEventRecord(c->ev_me[k], c->stream) != cudaSuccess ||
+        cudaStreamWaitEvent(c->sme_st, c->ev_me[k], 0) != cudaSuccess)
+      return launch_status();
+    if ((st = launch_sme(c, cf, sfs + k, mvs + 2 * off, sads + off, qmvs + 2 * off, qsads + off, 1, c->sme_st)) != ME_OK)
+      return st;
+  }
+  c->timing = saved;
+  if (cudaEventRecord(c->ev_sme_done, c->sme_st) != cudaSuccess ||
+      cudaStreamWaitEvent(c->stream, c->ev_sme_done, 0) != cudaSuccess)
+    return launch_status();
+  return ME_OK;
+}
+
 // ------------------------------------------------------------------ API ----
 extern "C" int me_estimate(me_ctx* c, const uint8_t* cf, const uint8_t* const* rfs, int16_t* out_mvs,
                            uint16_t* out_sads) {
@@ -378,9 +433,8 @@ extern "C" int me_encode_frame(me_ctx* c, const uint8_t* cf, const uint8_t* cons
   if (c->fuse)   // ME with the SME fused into the same CTAs (one launch)
     return launch_me(c, cf, rfs, out_mvs, out_sads, c->n_rf, c->stream, reinterpret_cast<const uint8_t* const*>(sfs),
                      out_qmvs, out_qsads);
-  if ((st = launch_me(c, cf, rfs, mvs, sads, c->n_rf, c->stream)) != ME_OK) return st;
-  return launch_sme(c, cf, reinterpret_cast<const uint8_t* const*>(sfs), mvs, sads, out_qmvs, out_qsads, c->n_rf,
-                    c->stream);
+  return run_me_sme(c, cf, rfs, reinterpret_cast<const uint8_t* const*>(sfs), mvs, sads, out_qmvs, out_qsads, c->n_rf,
+                    nullptr);
 }
 
 // ------------------------------------------------------------ IPPP stream ----
@@ -478,9 +532,7 @@ extern "C" int me_stream_push(me_ctx* c, const uint8_t* cf, int cf_on_host, int1
         return launch_status();
       if ((st = launch_int(c, new_rf, new_sf, c->side)) != ME_OK) return st;
       if (cudaEventRecord(c->ev_join, c->side) != cudaSuccess) return launch_status();
-      if ((st = launch_me(c, cur, rfs, c->d_mvs, c->d_sads, n_ref, c->stream)) != ME_OK) return st;
-      if (cudaStreamWaitEvent(c->stream, c->ev_join, 0) != cudaSuccess) return launch_status();
-      if ((st = launch_sme(c, cur, sfs, c->d_mvs, c->d_sads, qm, qs, n_ref, c->stream)) != ME_OK) return st;
+      if ((st = run_me_sme(c, cur, rfs, sfs, c->d_mvs, c->d_sads, qm, qs, n_ref, c->ev_join)) != ME_OK) return st;
     }
     const size_t nmv = (size_t)(c->row1 - c->row0) * c->mb_cols * c->n_rf * kNPart;
     if (cudaEventRecord(c->ev_done[par], c->stream) != cudaSuccess) return launch_status();
@@ -504,6 +556,7 @@ extern "C" int me_sync(me_ctx* c) {
   if (e == cudaSuccess && c->copy_in) e = cudaStreamSynchronize(c->copy_in);
   if (e == cudaSuccess && c->copy_out) e = cudaStreamSynchronize(c->copy_out);
   if (e == cudaSuccess && c->side) e = cudaStreamSynchronize(c->side);
+  if (e == cudaSuccess && c->sme_st) e = cudaStreamSynchronize(c->sme_st);
   return e == cudaSuccess ? ME_OK : ME_ECUDA;
 }
 
@@ -537,8 +590,17 @@ extern "C" int me_get_timings(me_ctx* c, float* ms_int, float* ms_me, float* ms_
   return ME_OK;
 }
 
-extern "C" int me_set_fused(me_ctx* c, int on) {
+extern "C" int me_set_option(me_ctx* c, int option, int value) {
   if (!c) return ME_EINVAL;
-  c->fuse = on ? 1 : 0;
-  return ME_OK;
+  switch (option) {
+    case ME_OPT_FUSED_SME: c->fuse = value ? 1 : 0; return ME_OK;
+    case ME_OPT_PIPELINE_RF: c->pipeline = value ? 1 : 0; return ME_OK;
+    case ME_OPT_ME_CTAS_PER_SM:
+      if (value < 0 || value > 32) return ME_EINVAL;
+      c->me_ctas_per_sm = value;
+      return ME_OK;
+    default: return ME_EINVAL;
+  }
 }
+
+extern "C" int me_set_fused(me_ctx* c, int on) { return me_set_option(c, ME_OPT_FUSED_SME, on); }
