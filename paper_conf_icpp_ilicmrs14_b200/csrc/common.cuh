@@ -17,22 +17,27 @@ __device__ __forceinline__ uint32_t vad4(uint32_t a, uint32_t b, uint32_t c) {
   return d;
 }
 
-// per-byte rounded average (u+v+1)>>1 on 4 packed bytes (VAVRG4)
+// per-byte rounded average (u+v+1)>>1 on 4 packed bytes.  PTX vavrg4 is NOT
+// native on sm_100a (ptxas expands it byte by byte, ~16 instructions), so use
+// the exact SWAR identity ceil((a+b)/2) = (a|b) - ((a^b)>>1) per byte; the mask
+// stops bit 0 of a byte from shifting into its neighbour, and the subtraction
+// never borrows across bytes because (a^b)>>1 <= a|b bytewise.  4 ALU ops.
 __device__ __forceinline__ uint32_t vavg4(uint32_t a, uint32_t b) {
-  uint32_t d;
-  asm("vavrg4.u32.u32.u32 %0, %1, %2, %3;" : "=r"(d) : "r"(a), "r"(b), "r"(0u));
-  return d;
+  return (a | b) - (((a ^ b) & 0xfefefefeu) >> 1);
 }
 
 __device__ __forceinline__ int clampi(int v, int lo, int hi) { return v < lo ? lo : (v > hi ? hi : v); }
 
 // Four bytes of row y of a W x H tight u8 frame starting at column x, with
-// coordinate clamping (G5).  Fast path: one aligned 32-bit load.
+// coordinate clamping (G5).  Fast paths: one aligned 32-bit load inside the
+// frame; one byte load broadcast when the 4 columns all clamp to the same edge.
 __device__ __forceinline__ uint32_t load4_clamped(const uint8_t* __restrict__ f, int W, int H, int x, int y) {
   y = clampi(y, 0, H - 1);
   const uint8_t* row = f + (size_t)y * W;
   if (x >= 0 && x + 3 < W && ((reinterpret_cast<uintptr_t>(row + x) & 3) == 0))
     return __ldg(reinterpret_cast<const uint32_t*>(row + x));
+  if (x + 3 <= 0) return 0x01010101u * __ldg(row);
+  if (x >= W - 1) return 0x01010101u * __ldg(row + W - 1);
   uint32_t v = 0;
 #pragma unroll
   for (int i = 0; i < 4; ++i) v |= (uint32_t)__ldg(row + clampi(x + i, 0, W - 1)) << (8 * i);

@@ -304,18 +304,16 @@ static int launch_int(me_ctx* c, const uint8_t* rf, uint8_t* sf, cudaStream_t st
     g_hi = std::max(g_lo, std::min(groups, (c->W - 20 + c->sf_pad) / 16 + 1));
   }
   P.g_lo = g_lo; P.g_hi = g_hi;
-  dim3 block(32, 4);
-  const int nrows = P.row_end - P.row_begin;
-  tmark(c, 0, st);
-  if (g_hi > g_lo) {
-    int_subpel_kernel<true><<<dim3((g_hi - g_lo + 31) / 32, (nrows + 3) / 4), block, 0, st>>>(P);
-    c->last_launches++;
-  }
   const int nb = groups - (g_hi - g_lo);
-  if (nb > 0) {
-    int_subpel_kernel<false><<<dim3((nb + 31) / 32, (nrows + 3) / 4), block, 0, st>>>(P);
-    c->last_launches++;
-  }
+  int bx = 1;
+  while (bx < nb && bx < 32) bx <<= 1;
+  P.border_bx = bx;
+  const int nrows = P.row_end - P.row_begin;
+  const dim3 block(32, 4);
+  const dim3 grid(std::max(1, (g_hi - g_lo + 31) / 32), (nrows + 3) / 4, nb > 0 ? 2 : 1);
+  tmark(c, 0, st);
+  int_subpel_kernel<<<grid, block, 0, st>>>(P);
+  c->last_launches++;
   tmark(c, 1, st);
   return launch_status();
 }

@@ -25,6 +25,7 @@ struct IntParams {
   int W, H, pad, pitch, rows, row_begin, row_end;
   size_t plane;   // bytes per phase plane = rows * pitch
   int g_lo, g_hi; // interior 16-column groups [g_lo, g_hi): every source word in-frame and aligned
+  int border_bx;  // border blocks: groups per block row (power of two >= number of border groups)
 };
 
 // Two columns per 32-bit register, one per 16-bit lane, and every lane kept
@@ -53,15 +54,12 @@ __device__ __forceinline__ uint32_t clip_j(int jb) { return (uint32_t)min(max(jb
 // low bytes of four u16 lanes (pairs a, b) -> one byte word
 __device__ __forceinline__ uint32_t bytes_of(uint32_t a, uint32_t b) { return __byte_perm(a, b, 0x6420); }
 
-// INTERIOR launch: groups [g_lo, g_hi) (no clamping code at all, warps never
-// diverge); border launch: the groups outside it, with per-byte clamping.
+// One launch, two kinds of blocks (uniform per block, so warps never diverge):
+// blockIdx.z == 1: interior groups [g_lo, g_hi) with no clamping code at all;
+// blockIdx.z == 0: the few border groups, 128 threads = border_bx groups x rows
+// (dispatched first: they are the latency-bound tail otherwise).
 template <bool INTERIOR>
-__global__ void __launch_bounds__(128) int_subpel_kernel(const IntParams P) {
-  const int t = blockIdx.x * blockDim.x + threadIdx.x;
-  const int nb_left = P.g_lo;
-  const int g = INTERIOR ? P.g_lo + t : (t < nb_left ? t : P.g_hi + (t - nb_left));   // 16-column group
-  const int rr = P.row_begin + blockIdx.y * blockDim.y + threadIdx.y;
-  if ((INTERIOR ? g >= P.g_hi : 16 * g >= P.pitch) || rr >= P.row_end) return;
+__device__ __forceinline__ void int_body(const IntParams& P, int g, int rr) {
   const int x0 = 16 * g - P.pad, y = rr - P.pad;
 
   // source rows y-2 .. y+3 (k = 0..5), columns x0-4 .. x0+19 (c = 0..23, 6 words)
@@ -176,6 +174,24 @@ __global__ void __launch_bounds__(128) int_subpel_kernel(const IntParams P) {
 #undef Pq_
 #undef Q_
 #undef R_
+}
+
+__global__ void __launch_bounds__(128) int_subpel_kernel(const IntParams P) {
+  if (blockIdx.z == gridDim.z - 1) {
+    const int g = P.g_lo + blockIdx.x * blockDim.x + threadIdx.x;
+    const int rr = P.row_begin + blockIdx.y * blockDim.y + threadIdx.y;
+    if (g < P.g_hi && rr < P.row_end) int_body<true>(P, g, rr);
+  } else {
+    if (blockIdx.x != 0) return;
+    const int t = threadIdx.y * blockDim.x + threadIdx.x;
+    const int bx = P.border_bx, by = (blockDim.x * blockDim.y) / bx;
+    const int tb = t % bx, tr = t / bx;
+    const int groups = P.pitch / 16, nb = groups - (P.g_hi - P.g_lo);
+    if (tb >= nb) return;
+    const int g = tb < P.g_lo ? tb : P.g_hi + (tb - P.g_lo);
+    const int rr = P.row_begin + blockIdx.y * by + tr;
+    if (rr < P.row_end) int_body<false>(P, g, rr);
+  }
 }
 
 }  // namespace feves
