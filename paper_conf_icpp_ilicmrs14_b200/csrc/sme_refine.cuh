@@ -78,6 +78,18 @@ __device__ __forceinline__ int mode_part(int bx, int by) {
 
 // YG = blocks of a partition along by inside the lane (1, 2, 4);
 // XMASK = the bx lane bits a partition spans (0, 1, 3).
+//
+// Half stage: the 8 candidates c + 2 s_k are half-grid samples, read from the
+// b / h / j planes (phases 2, 8, 10).  Quarter stage: the 8 neighbours of the
+// best half position H are, by the interpolation rule itself (O2: every
+// quarter sample is the rounded average of two half-grid samples), rounded
+// averages of the 3x3 half-grid samples around H.  Those 9 windows per row come
+// from the 4 planes G, b, h, j only (phases 0, 2, 8, 10), so the refinement
+// touches 4 of the 16 planes (4x less L1/L2 footprint); the averages are the
+// SWAR byte average, bit-identical to the quarter planes INT writes.
+// Axis neighbour (dx,0) = avg(HP(0,0), HP(dx,0)), (0,dy) likewise; diagonal
+// (dx,dy) = avg of the two corners of the half-grid unit square that have one
+// odd coordinate: (0,0) & (dx,dy) if H has mixed parity, else (dx,0) & (0,dy).
 template <int MODE, int YG, int XMASK>
 __device__ __forceinline__ void refine_mode(const SmeParams& P, const uint8_t* __restrict__ sf, size_t o, int bx,
                                             int xs, int ys0, bool writer, const uint32_t (&cfs)[16]) {
@@ -101,35 +113,76 @@ __device__ __forceinline__ void refine_mode(const SmeParams& P, const uint8_t* _
       best[g] = xsum<XMASK>(s);
     }
   }
-#pragma unroll
-  for (int stage = 0; stage < 2; ++stage) {
+  // ---- half stage (all 8 candidates' loads first: latency-bound) ----
+  {
     int ox[NG], oy[NG];
 #pragma unroll
-    for (int g = 0; g < NG; ++g) { ox[g] = bvx[g]; oy[g] = bvy[g]; }   // half: c; quarter: best half
-    // all 8 ring candidates' loads first (memory-level parallelism: the kernel
-    // is latency-bound), then the strictly ordered compare/updates
+    for (int g = 0; g < NG; ++g) { ox[g] = bvx[g]; oy[g] = bvy[g]; }
     uint32_t sad[8][NG];
 #pragma unroll
-    for (int k = 0; k < 8; ++k) {
-      const int sx = c_ring1[k][0] << (1 - stage), sy = c_ring1[k][1] << (1 - stage);
+    for (int k = 0; k < 8; ++k)
 #pragma unroll
       for (int g = 0; g < NG; ++g) {
         uint32_t t = 0;
 #pragma unroll
         for (int j = 0; j < YG; ++j)
-          t += strip_block_sad(sf, P.plane, P.pitch, P.pad, xs, ys0 + 4 * (g * YG + j), ox[g] + sx, oy[g] + sy,
-                               cfs + 4 * (g * YG + j));
+          t += strip_block_sad(sf, P.plane, P.pitch, P.pad, xs, ys0 + 4 * (g * YG + j), ox[g] + 2 * c_ring1[k][0],
+                               oy[g] + 2 * c_ring1[k][1], cfs + 4 * (g * YG + j));
         sad[k][g] = t;
       }
-    }
 #pragma unroll
-    for (int k = 0; k < 8; ++k) {
-      const int sx = c_ring1[k][0] << (1 - stage), sy = c_ring1[k][1] << (1 - stage);
+    for (int k = 0; k < 8; ++k)
 #pragma unroll
       for (int g = 0; g < NG; ++g) {
         const uint32_t t = xsum<XMASK>(sad[k][g]);
-        if (t < best[g]) { best[g] = t; bvx[g] = ox[g] + sx; bvy[g] = oy[g] + sy; }
+        if (t < best[g]) { best[g] = t; bvx[g] = ox[g] + 2 * c_ring1[k][0]; bvy[g] = oy[g] + 2 * c_ring1[k][1]; }
       }
+  }
+  // ---- quarter stage from the 3x3 half-grid windows around the best half position ----
+#pragma unroll
+  for (int g = 0; g < NG; ++g) {
+    const int hx = bvx[g] >> 1, hy = bvy[g] >> 1;          // half-grid coordinates (bvx, bvy even)
+    const bool mixed = ((hx ^ hy) & 1) != 0;
+    int off[3][3];                                          // window offsets from the strip's row base
+#pragma unroll
+    for (int b = 0; b < 3; ++b)
+#pragma unroll
+      for (int a = 0; a < 3; ++a)
+        off[b][a] = (8 * ((hy + b - 1) & 1) + 2 * ((hx + a - 1) & 1)) * (int)P.plane +
+                    ((hy + b - 1) >> 1) * P.pitch + ((hx + a - 1) >> 1);
+    uint32_t qs[8];
+#pragma unroll
+    for (int k = 0; k < 8; ++k) qs[k] = 0;
+    const uint8_t* rowp = sf + (size_t)(ys0 + 4 * g * YG + P.pad) * P.pitch + (xs + P.pad);
+#pragma unroll 1
+    for (int rr = 0; rr < 4 * YG; ++rr, rowp += P.pitch) {
+      uint32_t hp[3][3];
+#pragma unroll
+      for (int b = 0; b < 3; ++b)
+#pragma unroll
+        for (int a = 0; a < 3; ++a) {
+          const uintptr_t ad = reinterpret_cast<uintptr_t>(rowp + off[b][a]);
+          const uint32_t* w = reinterpret_cast<const uint32_t*>(ad & ~uintptr_t(3));
+          hp[b][a] = __funnelshift_r(__ldg(w), __ldg(w + 1), 8u * (uint32_t)(ad & 3));
+        }
+      const uint32_t c = load4_clamped(P.cf, P.W, P.H, xs, ys0 + 4 * g * YG + rr);   // L1 hit
+#pragma unroll
+      for (int k = 0; k < 8; ++k) {
+        const int dx = c_ring1[k][0], dy = c_ring1[k][1];
+        uint32_t smp;
+        if (dx == 0 || dy == 0) {
+          smp = vavg4(hp[1][1], hp[1 + dy][1 + dx]);
+        } else {
+          smp = vavg4(mixed ? hp[1][1] : hp[1][1 + dx], mixed ? hp[1 + dy][1 + dx] : hp[1 + dy][1]);
+        }
+        qs[k] = vad4(c, smp, qs[k]);
+      }
+    }
+    const int ox = bvx[g], oy = bvy[g];
+#pragma unroll
+    for (int k = 0; k < 8; ++k) {             // spiral order, strict < (G14)
+      const uint32_t t = xsum<XMASK>(qs[k]);
+      if (t < best[g]) { best[g] = t; bvx[g] = ox + c_ring1[k][0]; bvy[g] = oy + c_ring1[k][1]; }
     }
   }
   if (writer && (bx & XMASK) == 0) {     // partition leader lane writes
