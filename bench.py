@@ -205,6 +205,17 @@ def config_json(cfg, args):
 
 # --------------------------------------------------------------------- feves --
 
+def _all_max(x):
+    """max over ranks (device tensor for NCCL, host for the gloo smoke test)"""
+    import torch.distributed as dist
+    if dist.get_backend() == "gloo":
+        h = x.cpu()
+        dist.all_reduce(h, op=dist.ReduceOp.MAX)
+        return h
+    dist.all_reduce(x, op=dist.ReduceOp.MAX)
+    return x
+
+
 def run_feves(args, cfg):
     import torch
     import torch.distributed as dist
@@ -218,10 +229,15 @@ def run_feves(args, cfg):
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    local = local % torch.cuda.device_count()        # FEVES_DIST_BACKEND=gloo smoke test: ranks may share a GPU
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     if world > 1:
-        dist.init_process_group("nccl", device_id=dev)
+        backend = os.environ.get("FEVES_DIST_BACKEND", "nccl")
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=dev)
+        else:
+            dist.init_process_group(backend)
     me = feves.MotionEstimator(cfg.width, cfg.height, cfg.sa_range, cfg.n_rf, device=dev)
     r0, r1 = stripes(me.mb_rows, world)[rank]
     me.set_rows(r0, r1)
@@ -273,7 +289,7 @@ def run_feves(args, cfg):
     step_ms = [a.elapsed_time(b) for a, b in ev]
     tot = torch.tensor([sum(step_ms)], dtype=torch.float64, device=dev)
     if world > 1:
-        dist.all_reduce(tot, op=dist.ReduceOp.MAX)
+        tot = _all_max(tot)
         dist.barrier()
     total_ms = float(tot.item())
     fps = args.steps / (total_ms / 1e3)
@@ -346,7 +362,7 @@ def run_feves(args, cfg):
         e1.record(stream)
         torch.cuda.synchronize()
         tt = torch.tensor([e0.elapsed_time(e1)], dtype=torch.float64, device=dev)
-        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+        tt = _all_max(tt)
         e2e = {"value": args.e2e_steps / (float(tt.item()) / 1e3), "unit": "frames/s",
                "h2d_bytes_per_step": pinned[0].numel(),
                "d2h_bytes_per_step": qm_h.numel() * 2 + qs_h.numel() * 2,

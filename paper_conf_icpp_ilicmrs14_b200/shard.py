@@ -52,6 +52,11 @@ class ShardedStream:
         self.world = dist.get_world_size(group)
         self.max_rows = max(r1 - r0 for r0, r1 in stripes(backend.mb_rows, self.world))
 
+    def _host_staged(self, t):
+        # gloo has no CUDA gather: stage through the host (only used to smoke-test the
+        # multi-rank path on a single GPU; NCCL moves device buffers directly)
+        return dist.get_backend(self.group) == "gloo" and t.is_cuda
+
     def push(self, frame, frame_buf):
         """frame: this step's frame on rank ``src`` (any device tensor, ignored elsewhere);
         frame_buf: a same-shape buffer on every rank that receives it.
@@ -59,7 +64,12 @@ class ShardedStream:
         if self.rank == self.src:
             if frame.data_ptr() != frame_buf.data_ptr():
                 frame_buf.copy_(frame)
-        dist.broadcast(frame_buf, self.src, group=self.group)
+        if self._host_staged(frame_buf):
+            h = frame_buf.cpu()
+            dist.broadcast(h, self.src, group=self.group)
+            frame_buf.copy_(h)
+        else:
+            dist.broadcast(frame_buf, self.src, group=self.group)
         qm, qs, n_ref = self.be.stream_push(frame_buf)
         return self._gather(qm, qs, n_ref)
 
@@ -70,6 +80,9 @@ class ShardedStream:
         pad_s[: qs.shape[0]].copy_(qs)
         # one collective for both fields: view the int16/uint16 payloads as bytes
         payload = torch.cat([pad_m.view(torch.uint8).reshape(-1), pad_s.view(torch.uint8).reshape(-1)])
+        dev = payload.device
+        if self._host_staged(payload):
+            payload = payload.cpu()
         if self.rank == self.src:
             bufs = [torch.empty_like(payload) for _ in range(self.world)]
             dist.gather(payload, bufs, dst=self.src, group=self.group)
@@ -80,6 +93,6 @@ class ShardedStream:
                 s = b[nm:].view(torch.uint16).reshape(pad_s.shape)[: r1 - r0]
                 parts_m.append(m)
                 parts_s.append(s)
-            return torch.cat(parts_m), torch.cat(parts_s), n_ref
+            return torch.cat(parts_m).to(dev), torch.cat(parts_s).to(dev), n_ref
         dist.gather(payload, None, dst=self.src, group=self.group)
         return None

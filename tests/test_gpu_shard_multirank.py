@@ -1,0 +1,65 @@
+"""Multi-process MB-row sharding on the GPU path: 2 ranks (sharing cuda:0, gloo,
+CPU-staged collectives) run ShardedStream over real MotionEstimator stripes; rank 0's
+assembled quarter-pel MVs/SADs must equal a single-process full-frame stream, bitwise
+(P11 on the CUDA path, through the same code bench.py runs under torchrun)."""
+import os
+import socket
+
+import numpy as np
+import pytest
+import torch
+import torch.multiprocessing as mp
+
+pytestmark = pytest.mark.gpu
+
+W, H, S, N_RF, N_FRAMES = 160, 120, 32, 2, 5      # 8 MB rows, ragged bottom
+
+
+def _worker(rank, world, port, q):
+    import torch.distributed as dist
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        import paper_conf_icpp_ilicmrs14_b200 as F
+        from paper_conf_icpp_ilicmrs14_b200.shard import ShardedStream, stripes
+        from synth import gen_tex
+        torch.cuda.set_device(0)
+        me = F.MotionEstimator(W, H, S, N_RF)
+        r0, r1 = stripes(me.mb_rows, world)[rank]
+        me.set_rows(r0, r1)
+        ss = ShardedStream(me)
+        buf = torch.zeros(H, W, dtype=torch.uint8, device="cuda")
+        frames = [torch.from_numpy(gen_tex(W, H, t, 31)).cuda() for t in range(N_FRAMES)]
+        outs = []
+        for t in range(N_FRAMES):
+            r = ss.push(frames[t], buf)
+            if rank == 0:
+                outs.append((r[0].cpu().numpy(), r[1].cpu().numpy(), r[2]))
+        if rank == 0:
+            ref = F.MotionEstimator(W, H, S, N_RF)
+            refs = []
+            for t in range(N_FRAMES):
+                qm, qs, n = ref.stream_push(frames[t])
+                refs.append((qm.cpu().numpy(), qs.cpu().numpy(), n))
+            ok = all(np.array_equal(a[0][:, :, :a[2]], b[0][:, :, :b[2]]) and
+                     np.array_equal(a[1][:, :, :a[2]], b[1][:, :, :b[2]]) and a[2] == b[2]
+                     for a, b in zip(outs, refs))
+            q.put(ok)
+    finally:
+        dist.destroy_process_group()
+
+
+def test_two_rank_sharded_stream_equals_single():
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    with socket.socket() as s:
+        s.bind(("127.0.0.1", 0))
+        port = s.getsockname()[1]
+    procs = [ctx.Process(target=_worker, args=(r, 2, port, q)) for r in range(2)]
+    for p in procs:
+        p.start()
+    ok = q.get(timeout=600)
+    for p in procs:
+        p.join(timeout=120)
+        assert p.exitcode == 0
+    assert ok
