@@ -51,6 +51,7 @@ def parse():
     ap.add_argument("--pipeline", type=int, default=None, help="ME_OPT_PIPELINE_RF (default: library default)")
     ap.add_argument("--me-ctas", type=int, default=None, help="ME_OPT_ME_CTAS_PER_SM")
     ap.add_argument("--fused", type=int, default=None, help="ME_OPT_FUSED_SME")
+    ap.add_argument("--adaptive", action="store_true", help="N>1: re-split MB rows every frame (SURVEY §8 f3)")
     return ap.parse_args()
 
 
@@ -200,7 +201,8 @@ def run_reference(args, cfg):
 def config_json(cfg, args):
     return {"workload": cfg.name, "baseline_config_index": cfg.baseline_index, "width": cfg.width,
             "height": cfg.height, "n_rf": cfg.n_rf, "sa_range": cfg.sa_range, "path": "int+me+sme (IPPP stream)",
-            "partitions": 41, "parallelism": f"mb-row x{args.gpus}", "l2": "flushed (512 MiB write) before every timed step"}
+            "partitions": 41, "parallelism": f"mb-row x{args.gpus}" + (" adaptive" if args.adaptive else ""),
+            "l2": "flushed (512 MiB write) before every timed step"}
 
 
 # --------------------------------------------------------------------- feves --
@@ -240,7 +242,7 @@ def run_feves(args, cfg):
             dist.init_process_group(backend)
     me = feves.MotionEstimator(cfg.width, cfg.height, cfg.sa_range, cfg.n_rf, device=dev)
     r0, r1 = stripes(me.mb_rows, world)[rank]
-    me.set_rows(r0, r1)
+    me.set_rows(r0, r1)      # (ShardedStream may re-split later in adaptive mode)
     for opt, val in ((me.OPT_PIPELINE_RF, args.pipeline), (me.OPT_ME_CTAS_PER_SM, args.me_ctas),
                      (me.OPT_FUSED_SME, args.fused)):
         if val is not None:
@@ -254,7 +256,7 @@ def run_feves(args, cfg):
     pinned = [torch.from_numpy(f).pin_memory() for f in host]
     buf = torch.empty_like(frames[0])
     flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
-    ss = ShardedStream(me) if world > 1 else None
+    ss = ShardedStream(me, adaptive=args.adaptive) if world > 1 else None
 
     def push(t):
         if ss is not None:
@@ -324,7 +326,7 @@ def run_feves(args, cfg):
     me_ms = statistics.mean(m[1] for m in mod)              # fused: ME + SME in one kernel
     sme_ms = None if fused else statistics.mean(m[2] for m in mod)
     me_only_ms = statistics.mean(me_only)
-    stripe_frac = (r1 - r0) / me.mb_rows
+    stripe_frac = (me.row1 - me.row0) / me.mb_rows
     pk, pk_src = peaks()
     peak_px = N_SM * PX_PER_CLK_SM * pk.get("sm_max_mhz", 1965.0) * 1e6
     dom_px = (u["me_px"] + (u["sme_px"] if fused else 0)) * stripe_frac

@@ -61,6 +61,7 @@ struct me_ctx {
   int me_ctas_per_sm;    // cap on resident ME CTAs per SM (0 = hardware maximum; ME_OPT_ME_CTAS_PER_SM)
   cudaStream_t sme_st;   // pipeline: SME stream
   cudaEvent_t ev_me[kMaxRf], ev_sme_done;
+  int sf_v0[kMaxRf], sf_v1[kMaxRf];   // MB rows whose SF rows each SF-ring slot holds (re-split support)
 };
 
 static thread_local int g_last_error = ME_OK;
@@ -514,6 +515,21 @@ extern "C" int me_stream_push(me_ctx* c, const uint8_t* cf, int cf_on_host, int1
     for (int k = 0; k < n_ref; ++k) {           // ref_idx k = frame t-1-k
       rfs[k] = c->ring + (size_t)((t - 1 - k) % slots) * fb;
       sfs[k] = c->sf_ring + (size_t)((t - 1 - k) % c->n_rf) * sb;
+    }
+    // f3 re-split: an SF computed for another stripe may lack rows this stripe reads;
+    // recompute it from the frame ring (the ring holds whole frames) before ME/SME
+    for (int k = 1; k < n_ref; ++k) {
+      const int slot = (int)((t - 1 - k) % c->n_rf);
+      if (!(c->sf_v0[slot] <= c->row0 && c->row1 <= c->sf_v1[slot])) {
+        if ((st = launch_int(c, rfs[k], c->sf_ring + (size_t)slot * sb, c->stream)) != ME_OK) return st;
+        c->sf_v0[slot] = c->row0;
+        c->sf_v1[slot] = c->row1;
+      }
+    }
+    {
+      const int slot = (int)((t - 1) % c->n_rf);   // INT of the newest RF below covers this stripe
+      c->sf_v0[slot] = c->row0;
+      c->sf_v1[slot] = c->row1;
     }
     int16_t* qm = (out_qmvs && !out_on_host) ? out_qmvs : (out_on_host ? c->d_qmvs2[par] : c->d_qmvs);
     uint16_t* qs = (out_qsads && !out_on_host) ? out_qsads : (out_on_host ? c->d_qsads2[par] : c->d_qsads);

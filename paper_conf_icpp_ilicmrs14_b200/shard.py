@@ -35,22 +35,96 @@ def stripes(n_rows: int, g: int):
     return out
 
 
+def split_rows(n_rows: int, weights):
+    """Contiguous stripes with sizes proportional to ``weights`` (largest-remainder
+    rounding, at least one row each): the m_i of eq. (1), sum m_i = N."""
+    g = len(weights)
+    tot = float(sum(weights))
+    raw = [n_rows * w / tot for w in weights]
+    m = [max(1, int(r)) for r in raw]
+    while sum(m) > n_rows:                      # min-1 clamps can overshoot
+        i = max((k for k in range(g) if m[k] > 1), key=lambda k: m[k] - raw[k])
+        m[i] -= 1
+    rem = sorted(range(g), key=lambda k: raw[k] - m[k], reverse=True)
+    i = 0
+    while sum(m) < n_rows:
+        m[rem[i % g]] += 1
+        i += 1
+    out, r0 = [], 0
+    for k in range(g):
+        out.append((r0, r0 + m[k]))
+        r0 += m[k]
+    return out
+
+
+class AdaptiveSplit:
+    """Adaptive MB-row distribution: the paper's Framework Control
+    (Alg. 1) on identical GPUs.  Frame 1 is split equidistantly; after
+    each frame the Performance Characterization K_i = (time of device i) / (rows of
+    device i) ("processing time per MB row") is updated, and the next split
+    minimises max_i K_i m_i subject to sum m_i = N -- the optimum of Alg. 2's LP when
+    only the ME/INT/SME rows are distributed -- i.e. m_i proportional to 1/K_i.
+    ``smoothing`` is an exponential average of K (absorbs timer noise; a real change
+    is tracked within a few frames)."""
+
+    def __init__(self, n_rows: int, world: int, smoothing: float = 0.5):
+        self.n_rows, self.world, self.alpha = n_rows, world, smoothing
+        self.cur = stripes(n_rows, world)
+        self.K = None
+
+    def stripes(self):
+        return list(self.cur)
+
+    def update(self, times):
+        rows = [r1 - r0 for r0, r1 in self.cur]
+        k_now = [max(t, 1e-9) / max(m, 1) for t, m in zip(times, rows)]
+        self.K = k_now if self.K is None else [self.alpha * a + (1 - self.alpha) * b
+                                               for a, b in zip(self.K, k_now)]
+        self.cur = split_rows(self.n_rows, [1.0 / k for k in self.K])
+        return self.stripes()
+
+
 def halo_rows(r0: int, r1: int, sa_range: int, height: int):
     """Frame rows a stripe [r0, r1) reads: [16 r0 - R - 3, 16 r1 + R + 3) clamped."""
     R = sa_range // 2
     return max(0, 16 * r0 - R - 3), min(height, 16 * r1 + R + 3)
 
 
-class ShardedStream:
-    """IPPP stream over G ranks: broadcast in, per-rank stripe push, gather out."""
+def cuda_event_timer(fn):
+    """(fn(), seconds) measured with CUDA events on the current stream: the per-device
+    execution time the Performance Characterization uses."""
+    a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    a.record()
+    out = fn()
+    b.record()
+    b.synchronize()
+    return out, a.elapsed_time(b) / 1e3
 
-    def __init__(self, backend, group=None, src: int = 0):
+
+class ShardedStream:
+    """IPPP stream over G ranks: broadcast in, per-rank stripe push, gather out.
+
+    With ``adaptive=True`` the stripes are re-split after every frame from the per-rank
+    stripe times (AdaptiveSplit); results do not depend on the split
+    (pin P11), the library recomputes the SF rows a new stripe needs."""
+
+    def __init__(self, backend, group=None, src: int = 0, adaptive: bool = False, timer=None):
         self.be = backend
         self.group = group
         self.src = src
         self.rank = dist.get_rank(group)
         self.world = dist.get_world_size(group)
-        self.max_rows = max(r1 - r0 for r0, r1 in stripes(backend.mb_rows, self.world))
+        self.split = AdaptiveSplit(backend.mb_rows, self.world) if adaptive else None
+        self.timer = timer or cuda_event_timer  # callable(fn) -> (result, seconds) for the stripe work
+        self.history = []                       # stripes used per frame (adaptive mode)
+        self._apply(self.split.stripes() if adaptive else stripes(backend.mb_rows, self.world))
+
+    def _apply(self, st):
+        self.cur = st
+        r0, r1 = st[self.rank]
+        if (getattr(self.be, "row0", None), getattr(self.be, "row1", None)) != (r0, r1):
+            self.be.set_rows(r0, r1)
+        self.max_rows = max(b - a for a, b in st)
 
     def _host_staged(self, t):
         # gloo has no CUDA gather: stage through the host (only used to smoke-test the
@@ -70,8 +144,17 @@ class ShardedStream:
             frame_buf.copy_(h)
         else:
             dist.broadcast(frame_buf, self.src, group=self.group)
-        qm, qs, n_ref = self.be.stream_push(frame_buf)
-        return self._gather(qm, qs, n_ref)
+        if self.split is None:
+            qm, qs, n_ref = self.be.stream_push(frame_buf)
+            return self._gather(qm, qs, n_ref)
+        (qm, qs, n_ref), secs = self.timer(lambda: self.be.stream_push(frame_buf))
+        out = self._gather(qm, qs, n_ref)
+        tdev = torch.device("cpu") if (dist.get_backend(self.group) == "gloo") else frame_buf.device
+        times = [torch.zeros(1, dtype=torch.float64, device=tdev) for _ in range(self.world)]
+        dist.all_gather(times, torch.tensor([secs], dtype=torch.float64, device=tdev), group=self.group)
+        self.history.append(self.cur)
+        self._apply(self.split.update([float(x) for x in times]))
+        return out
 
     def _gather(self, qm, qs, n_ref):
         pad_m = qm.new_zeros((self.max_rows,) + tuple(qm.shape[1:]))
@@ -88,7 +171,7 @@ class ShardedStream:
             dist.gather(payload, bufs, dst=self.src, group=self.group)
             parts_m, parts_s = [], []
             nm = pad_m.numel() * 2
-            for (r0, r1), b in zip(stripes(self.be.mb_rows, self.world), bufs):
+            for (r0, r1), b in zip(self.cur, bufs):
                 m = b[:nm].view(torch.int16).reshape(pad_m.shape)[: r1 - r0]
                 s = b[nm:].view(torch.uint16).reshape(pad_s.shape)[: r1 - r0]
                 parts_m.append(m)

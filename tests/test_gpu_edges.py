@@ -96,3 +96,24 @@ def test_many_contexts_and_streams(feves, orc):
         s.synchronize()
         np.testing.assert_array_equal(sa.cpu().numpy().reshape(-1, 1, 41), o_s)
         me.close()
+
+
+def test_stream_resplit_recomputes_sf(feves):
+    """f3: changing the stripe between pushes (as the adaptive split does) keeps results
+    identical to the full-frame stream: SFs computed for the old stripe are refreshed."""
+    W, H, S, n_rf = 64, 128, 16, 3                      # 8 MB rows
+    frames = [gen_tex(W, H, t, 13) for t in range(7)]
+    full = feves.MotionEstimator(W, H, S, n_rf)
+    ref = [full.stream_push(_dev(f)) for f in frames]
+    torch.cuda.synchronize()
+    me = feves.MotionEstimator(W, H, S, n_rf)
+    splits = [(0, 4), (0, 4), (0, 6), (2, 8), (0, 3), (5, 8), (1, 7)]
+    for t, (f, (r0, r1)) in enumerate(zip(frames, splits)):
+        me.set_rows(r0, r1)
+        q, qs, used = me.stream_push(_dev(f))
+        torch.cuda.synchronize()
+        if used:
+            assert torch.equal(q[:, :, :used], ref[t][0][r0:r1, :, :used]), (t, r0, r1)
+            assert torch.equal(qs[:, :, :used], ref[t][1][r0:r1, :, :used]), (t, r0, r1)
+    me.close()
+    full.close()

@@ -15,7 +15,17 @@ pytestmark = pytest.mark.gpu
 W, H, S, N_RF, N_FRAMES = 160, 120, 32, 2, 5      # 8 MB rows, ragged bottom
 
 
-def _worker(rank, world, port, q):
+class _SlowRank1:
+    def __init__(self, rank, be):
+        self.rank, self.be = rank, be
+
+    def __call__(self, fn):
+        out = fn()
+        torch.cuda.synchronize()
+        return out, (3.0 if self.rank == 1 else 1.0) * (self.be.row1 - self.be.row0)
+
+
+def _worker(rank, world, port, q, adaptive=False):
     import torch.distributed as dist
     os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
     dist.init_process_group("gloo", rank=rank, world_size=world)
@@ -27,7 +37,7 @@ def _worker(rank, world, port, q):
         me = F.MotionEstimator(W, H, S, N_RF)
         r0, r1 = stripes(me.mb_rows, world)[rank]
         me.set_rows(r0, r1)
-        ss = ShardedStream(me)
+        ss = ShardedStream(me, adaptive=adaptive, timer=_SlowRank1(rank, me) if adaptive else None)
         buf = torch.zeros(H, W, dtype=torch.uint8, device="cuda")
         frames = [torch.from_numpy(gen_tex(W, H, t, 31)).cuda() for t in range(N_FRAMES)]
         outs = []
@@ -44,22 +54,25 @@ def _worker(rank, world, port, q):
             ok = all(np.array_equal(a[0][:, :, :a[2]], b[0][:, :, :b[2]]) and
                      np.array_equal(a[1][:, :, :a[2]], b[1][:, :, :b[2]]) and a[2] == b[2]
                      for a, b in zip(outs, refs))
-            q.put(ok)
+            q.put((ok, ss.history))
     finally:
         dist.destroy_process_group()
 
 
-def test_two_rank_sharded_stream_equals_single():
+@pytest.mark.parametrize("adaptive", [False, True])
+def test_two_rank_sharded_stream_equals_single(adaptive):
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     with socket.socket() as s:
         s.bind(("127.0.0.1", 0))
         port = s.getsockname()[1]
-    procs = [ctx.Process(target=_worker, args=(r, 2, port, q)) for r in range(2)]
+    procs = [ctx.Process(target=_worker, args=(r, 2, port, q, adaptive)) for r in range(2)]
     for p in procs:
         p.start()
-    ok = q.get(timeout=600)
+    ok, history = q.get(timeout=600)
     for p in procs:
         p.join(timeout=120)
         assert p.exitcode == 0
     assert ok
+    if adaptive:                       # rank 1 reported 3x the time per row: rows moved to rank 0
+        assert history[0] == [(0, 4), (4, 8)] and history[-1] == [(0, 6), (6, 8)]

@@ -114,3 +114,122 @@ def test_stripes_and_halo():
     assert stripes(68, 2) == [(0, 34), (34, 68)]
     assert halo_rows(0, 9, 64, 1080) == (0, 144 + 35)
     assert halo_rows(60, 68, 64, 1080) == (960 - 35, 1080)
+
+
+# ------------------------------------------------------------- f3: adaptive split --
+
+def test_split_rows_properties():
+    from paper_conf_icpp_ilicmrs14_b200.shard import split_rows, stripes
+    assert split_rows(68, [1] * 8) == stripes(68, 8)
+    for n, w in [(68, [1, 2]), (135, [3, 1, 1, 5, 2, 2, 1, 1]), (5, [100, 1, 1]), (8, [1] * 8)]:
+        st = split_rows(n, w)
+        assert st[0][0] == 0 and st[-1][1] == n
+        assert all(a < b for a, b in st) and all(st[i][1] == st[i + 1][0] for i in range(len(st) - 1))
+    st = split_rows(90, [2, 1])
+    assert [b - a for a, b in st] == [60, 30]
+
+
+def test_adaptive_split_converges_to_inverse_cost():
+    from paper_conf_icpp_ilicmrs14_b200.shard import AdaptiveSplit
+    cost = [1.0, 3.0, 1.0]                    # time per MB row on each device
+    a = AdaptiveSplit(60, 3, smoothing=0.0)
+    for _ in range(3):
+        st = a.stripes()
+        a.update([cost[i] * (b - e) for i, (e, b) in enumerate(st)])
+    rows = [b - e for e, b in a.stripes()]
+    assert rows == [26, 8, 26] or rows == [26, 9, 25] or rows == [25, 9, 26], rows   # 60 * (1, 1/3, 1) / (7/3)
+    assert max(c * m for c, m in zip(cost, rows)) < max(c * 20 for c in cost)          # beats equidistant
+
+
+class SlowRankTimer:
+    """stripe 'time' = rows x per-rank cost (rank 1 is 3x slower): a deterministic stand-in
+    for the CUDA-event timer, so the test is about the control loop, not the host clock."""
+
+    def __init__(self, rank, backend):
+        self.rank, self.be = rank, backend
+
+    def __call__(self, fn):
+        out = fn()
+        return out, (3.0 if self.rank == 1 else 1.0) * (self.be.row1 - self.be.row0)
+
+
+def _adaptive_worker(rank, world, port, q):
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        from paper_conf_icpp_ilicmrs14_b200.shard import ShardedStream, stripes
+        mbr = -(-H2 // 16)
+        be = OracleStripeBackend2(*stripes(mbr, world)[rank])
+        ss = ShardedStream(be, adaptive=True, timer=SlowRankTimer(rank, be))
+        frames = [gen_tex(W2, H2, t, 9) for t in range(N2)]
+        buf = torch.zeros(H2, W2, dtype=torch.uint8)
+        outs = []
+        for t in range(N2):
+            r = ss.push(torch.from_numpy(frames[t]) if rank == 0 else buf, buf)
+            if rank == 0:
+                outs.append((r[0].numpy(), r[1].numpy(), r[2]))
+        if rank == 0:
+            q.put((outs, ss.history))
+    finally:
+        dist.destroy_process_group()
+
+
+W2, H2, N2 = 32, 128, 5          # 8 MB rows
+
+
+class OracleStripeBackend2(OracleStripeBackend):
+    """as OracleStripeBackend but on the W2 x H2 frames and re-splittable (set_rows)"""
+
+    def __init__(self, r0, r1):
+        super().__init__(r0, r1)
+        self.mb_cols, self.mb_rows = -(-W2 // 16), -(-H2 // 16)
+
+    def set_rows(self, r0, r1):
+        self.row0, self.row1 = r0, r1
+
+    def stream_push(self, frame):
+        from paper_conf_icpp_ilicmrs14_b200.shard import halo_rows
+        f = frame.numpy().copy()
+        t = len(self.ring)
+        self.ring.append(f)                     # whole frames (as the CUDA ring)
+        n_ref = min(t, N_RF)
+        qm = torch.zeros(self.mv_shape() + (2,), dtype=torch.int16)
+        qs = torch.zeros(self.mv_shape(), dtype=torch.uint16)
+        if n_ref:
+            lo, hi = halo_rows(self.row0, self.row1, S, H2)
+            def view(g):                         # only stripe + halo rows are trusted
+                g = g.copy(); g[:lo] = 7; g[hi:] = 250
+                return g
+            rfs = [view(self.ring[t - 1 - k]) for k in range(n_ref)]
+            mbs = np.arange(self.row0 * self.mb_cols, self.row1 * self.mb_cols, dtype=np.int32)
+            mv, _ = self.orc.me(view(f), rfs, S, mb_list=mbs)
+            q, s = self.orc.sme(view(f), rfs, mv, mb_list=mbs)
+            rows = self.row1 - self.row0
+            qm[:, :, :n_ref] = torch.from_numpy(q.reshape(rows, self.mb_cols, n_ref, 41, 2))
+            qs[:, :, :n_ref] = torch.from_numpy(s.reshape(rows, self.mb_cols, n_ref, 41))
+        return qm, qs, n_ref
+
+
+def test_adaptive_sharded_stream_moves_rows_and_stays_exact(orc):
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_adaptive_worker, args=(r, 2, port, q)) for r in range(2)]
+    for p in procs:
+        p.start()
+    outs, history = q.get(timeout=600)
+    for p in procs:
+        p.join(timeout=120)
+        assert p.exitcode == 0
+    assert history[0] == [(0, 4), (4, 8)]                  # equidistant first frame (P:68)
+    assert history[-1][0][1] - history[-1][0][0] == 6      # rank 1 is 3x slower -> 6 / 2 rows
+    frames = [gen_tex(W2, H2, t, 9) for t in range(N2)]
+    n = (-(-W2 // 16)) * (-(-H2 // 16))
+    for t, (qm, qs, n_ref) in enumerate(outs):
+        if n_ref == 0:
+            continue
+        rfs = [frames[t - 1 - k] for k in range(n_ref)]
+        mv, _ = orc.me(frames[t], rfs, S)
+        oq, os_ = orc.sme(frames[t], rfs, mv)
+        np.testing.assert_array_equal(qm.reshape(n, N_RF, 41, 2)[:, :n_ref], oq)
+        np.testing.assert_array_equal(qs.reshape(n, N_RF, 41)[:, :n_ref], os_)
