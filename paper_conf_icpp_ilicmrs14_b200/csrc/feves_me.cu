@@ -336,7 +336,7 @@ static int launch_sme(me_ctx* c, const uint8_t* cf, const uint8_t* const* sfs, c
   P.plane = (size_t)c->sf_rows * c->sf_pitch;
   const int warps = n_ref * P.n_rows * P.groups;
   tmark(c, 4, st);
-  sme_refine_kernel<<<(warps + 3) / 4, 128, 0, st>>>(P);
+  sme_refine_kernel<<<dim3((warps + 3) / 4, 7), 128, 0, st>>>(P);   // y = partition mode
   tmark(c, 5, st);
   c->last_launches++;
   return launch_status();

@@ -214,13 +214,15 @@ __global__ void __launch_bounds__(128) sme_refine_kernel(const SmeParams P) {
   for (int r = 0; r < 16; ++r) cfs[r] = load4_clamped(P.cf, P.W, P.H, xs, ys0 + r);
   const uint8_t* __restrict__ sf = P.sf[ref];
   const size_t o = ((size_t)(mrow * P.mb_cols + mbx) * P.rf_stride + ref) * kNPart;
-  refine_mode<0, 4, 3>(P, sf, o, bx, xs, ys0, writer, cfs);   // 16x16
-  refine_mode<1, 2, 3>(P, sf, o, bx, xs, ys0, writer, cfs);   // 16x8
-  refine_mode<2, 4, 1>(P, sf, o, bx, xs, ys0, writer, cfs);   // 8x16
-  refine_mode<3, 2, 1>(P, sf, o, bx, xs, ys0, writer, cfs);   // 8x8
-  refine_mode<4, 1, 1>(P, sf, o, bx, xs, ys0, writer, cfs);   // 8x4
-  refine_mode<5, 2, 0>(P, sf, o, bx, xs, ys0, writer, cfs);   // 4x8
-  refine_mode<6, 1, 0>(P, sf, o, bx, xs, ys0, writer, cfs);   // 4x4
+  switch (blockIdx.y) {   // one mode per warp: 7x the independent warps (the kernel is latency-bound)
+    case 0: refine_mode<0, 4, 3>(P, sf, o, bx, xs, ys0, writer, cfs); break;   // 16x16
+    case 1: refine_mode<1, 2, 3>(P, sf, o, bx, xs, ys0, writer, cfs); break;   // 16x8
+    case 2: refine_mode<2, 4, 1>(P, sf, o, bx, xs, ys0, writer, cfs); break;   // 8x16
+    case 3: refine_mode<3, 2, 1>(P, sf, o, bx, xs, ys0, writer, cfs); break;   // 8x8
+    case 4: refine_mode<4, 1, 1>(P, sf, o, bx, xs, ys0, writer, cfs); break;   // 8x4
+    case 5: refine_mode<5, 2, 0>(P, sf, o, bx, xs, ys0, writer, cfs); break;   // 4x8
+    default: refine_mode<6, 1, 0>(P, sf, o, bx, xs, ys0, writer, cfs); break;  // 4x4
+  }
 }
 
 }  // namespace feves

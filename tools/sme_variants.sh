@@ -1,4 +1,4 @@
 cd $GRAFT_REPO_ROOT
-for f in tools/sme_*.so; do
-  FEVES_LIB=$PWD/$f python bench.py --steps 30 --warmup 3 --no-e2e --no-cpu-baseline 2>/dev/null | python -c "import json,sys; d=json.load(sys.stdin); print('$f', round(d['kernels_ms']['sme']*1000,1), 'us sme', round(d['value'],1), 'fps')"
+for f in tools/smehb_*.so; do
+  FEVES_LIB=$PWD/$f python bench.py --steps 40 --warmup 3 --no-e2e --no-cpu-baseline 2>/dev/null | python -c "import json,sys; d=json.load(sys.stdin); print('$f', round(d['kernels_ms']['sme']*1000,1), 'us sme', round(d['value'],1), 'fps')"
 done
