@@ -11,6 +11,8 @@ arithmetic step of the method lives in that C file, which cites the passage of
 
   spiral_rank        G4                P1, P10 (closed form vs enumeration)
   me                 O1  (P:6)         P1 hand-computed, P2, P3, P4, P9 NumPy brute force
+  me(lam>0), sme(lam>0)  G18 (f4)      P12 hand-computed rate pins, P13 NumPy brute force
+  mode_decision      O4  (f2)    P14 closed forms, P13 NumPy enumeration
   sample/int_planes  O2  (P:6)  P5 closed forms + golden, P6, P7, P9
   sme                O3  (P:6)   P2, P8 (incl. half-pel synthetic), P9
 """
@@ -48,7 +50,12 @@ def lib():
         P = ctypes.c_void_p
         i = ctypes.c_int
         L.oracle_me.argtypes = [P, P, i, i, i, i, i, P, i, P, P, i]
+        L.oracle_me_rd.argtypes = [P, P, i, i, i, i, i, i, P, i, P, P, i]
         L.oracle_sme.argtypes = [P, P, i, i, i, P, i, P, P, P, i]
+        L.oracle_sme_rd.argtypes = [P, P, i, i, i, i, P, i, P, P, P, i]
+        L.oracle_mode_decision.argtypes = [P, P, i, i, i, P]
+        L.oracle_mv_bits.argtypes = [i, i]
+        L.oracle_mv_bits.restype = i
         L.oracle_int_planes.argtypes = [P, i, i, i, i, i, i, i, P, i]
         for fn in ("oracle_sample", "oracle_b1", "oracle_h1", "oracle_j1",
                    "oracle_j_horizontal_first", "oracle_ref_px"):
@@ -96,8 +103,9 @@ def all_mbs(W: int, H: int, row_begin: int = 0, row_end: int | None = None):
     return np.arange(row_begin * mb_cols, row_end * mb_cols, dtype=np.int32)
 
 
-def me(cf, rfs, sa_range: int, mb_list=None, sa_inclusive: bool = False, threads: int = 0):
-    """O1. Returns (mvs int16 [n_mb, n_rf, 41, 2], sads uint16 [n_mb, n_rf, 41])."""
+def me(cf, rfs, sa_range: int, mb_list=None, sa_inclusive: bool = False, threads: int = 0, lam: int = 0):
+    """O1 (lam > 0: cost J = SAD + lam * R(mv), G18). Returns (mvs int16 [n_mb, n_rf, 41, 2],
+    sads uint16 [n_mb, n_rf, 41]) -- the SAD of the chosen MV."""
     cf = _u8(cf)
     rfs = [_u8(r) for r in rfs]
     H, W = cf.shape
@@ -105,15 +113,16 @@ def me(cf, rfs, sa_range: int, mb_list=None, sa_inclusive: bool = False, threads
     n = len(mb_list)
     mvs = np.zeros((n, len(rfs), N_PART, 2), np.int16)
     sads = np.zeros((n, len(rfs), N_PART), np.uint16)
-    rc = lib().oracle_me(_ptr(cf), _ptr_array(rfs), W, H, sa_range, len(rfs), int(sa_inclusive),
-                         _ptr(mb_list), n, _ptr(mvs), _ptr(sads), threads)
+    rc = lib().oracle_me_rd(_ptr(cf), _ptr_array(rfs), W, H, sa_range, len(rfs), int(sa_inclusive), int(lam),
+                            _ptr(mb_list), n, _ptr(mvs), _ptr(sads), threads)
     if rc != 0:
         raise ValueError("oracle_me: bad arguments")
     return mvs, sads
 
 
-def sme(cf, rfs, in_mvs, mb_list=None, threads: int = 0):
-    """O3. in_mvs int16 [n_mb, n_rf, 41, 2] full-pel. Returns (qmvs, sads)."""
+def sme(cf, rfs, in_mvs, mb_list=None, threads: int = 0, lam: int = 0):
+    """O3 (lam > 0: cost J = SAD + lam * R(qmv), G18). in_mvs int16 [n_mb, n_rf, 41, 2]
+    full-pel. Returns (qmvs, sads)."""
     cf = _u8(cf)
     rfs = [_u8(r) for r in rfs]
     H, W = cf.shape
@@ -122,11 +131,27 @@ def sme(cf, rfs, in_mvs, mb_list=None, threads: int = 0):
     in_mvs = np.ascontiguousarray(in_mvs, np.int16).reshape(n, len(rfs), N_PART, 2)
     qmvs = np.zeros((n, len(rfs), N_PART, 2), np.int16)
     sads = np.zeros((n, len(rfs), N_PART), np.uint16)
-    rc = lib().oracle_sme(_ptr(cf), _ptr_array(rfs), W, H, len(rfs), _ptr(mb_list), n,
-                          _ptr(in_mvs), _ptr(qmvs), _ptr(sads), threads)
+    rc = lib().oracle_sme_rd(_ptr(cf), _ptr_array(rfs), W, H, len(rfs), int(lam), _ptr(mb_list), n,
+                             _ptr(in_mvs), _ptr(qmvs), _ptr(sads), threads)
     if rc != 0:
         raise ValueError("oracle_sme: bad arguments")
     return qmvs, sads
+
+
+def mv_bits(qx: int, qy: int) -> int:
+    """G18 R(mv): se(v) Exp-Golomb bits of the quarter-pel MV components."""
+    return lib().oracle_mv_bits(qx, qy)
+
+
+def mode_decision(qmvs, sads, lam: int):
+    """O4: per MB [mb_type, sub_type x4, ref per 8x8 x4, cost] int32 [n_mb, 10]."""
+    qmvs = np.ascontiguousarray(qmvs, np.int16)
+    sads = np.ascontiguousarray(sads, np.uint16)
+    n, n_rf = sads.shape[0], sads.shape[1]
+    out = np.zeros((n, 10), np.int32)
+    if lib().oracle_mode_decision(_ptr(qmvs), _ptr(sads), n, n_rf, int(lam), _ptr(out)) != 0:
+        raise ValueError("oracle_mode_decision: bad arguments")
+    return out
 
 
 def sample(rf, X: int, Y: int) -> int:

@@ -129,16 +129,32 @@ int oracle_ref_px(const uint8_t *f, int W, int H, int x, int y) { return ref_px(
 
 /* CF is sampled the same way (its padding rows/cols replicate, G6). */
 
+/* --------------------------------------------------------------- G18 --
+ * Optional rate term (JM-style motion cost; the paper's ME text,
+ * P:6, names only the SAD -- lambda = 0 is the default reading G3):
+ *   J = SAD + lambda * R(mv),  R(mv) = se(mv.x) + se(mv.y) Exp-Golomb bits of
+ *   the quarter-pel MV against the zero predictor (G2: no MV predictor),
+ *   se(v): codeNum k = 2v-1 (v > 0) or -2v (v <= 0), bits = 2*floor(log2(k+1)) + 1. */
+static int se_bits(int v)
+{
+    unsigned k = v > 0 ? 2u * (unsigned)v - 1u : 2u * (unsigned)(-v);
+    int n = 0;
+    while ((k + 1u) >> (n + 1)) ++n;          /* n = floor(log2(k+1)) */
+    return 2 * n + 1;
+}
+
+int oracle_mv_bits(int qx, int qy) { return se_bits(qx) + se_bits(qy); }
+
 /* ------------------------------------------------------------------ O1 --
  * Integer FSBM ME for the MBs listed in mb_list (indices mby*mb_cols+mbx)
  * over n_rf RFs.  Outputs are written at position i of the list:
  *   out_mvs [n_mb][n_rf][41][2] int16 (dx, dy) full-pel
  *   out_sads[n_mb][n_rf][41]    uint16
  * Returns 0, or -1 on bad arguments.                                      */
-int oracle_me(const uint8_t *cf, const uint8_t *const *rfs, int W, int H,
-              int S, int n_rf, int sa_inclusive,
-              const int32_t *mb_list, int n_mb,
-              int16_t *out_mvs, uint16_t *out_sads, int n_threads)
+int oracle_me_rd(const uint8_t *cf, const uint8_t *const *rfs, int W, int H,
+                 int S, int n_rf, int sa_inclusive, int lambda,
+                 const int32_t *mb_list, int n_mb,
+                 int16_t *out_mvs, uint16_t *out_sads, int n_threads)
 {
     if (W <= 0 || H <= 0 || S < 2 || (S & 1) || n_rf < 1) return -1;
     int mb_cols = (W + 15) / 16;
@@ -158,7 +174,7 @@ int oracle_me(const uint8_t *cf, const uint8_t *const *rfs, int W, int H,
                 int ox, oy, w, h;
                 partition_geom(p, &ox, &oy, &w, &h);
                 int x0 = 16 * mbx + ox, y0 = 16 * mby + oy;
-                long best = -1; int bdx = 0, bdy = 0;
+                long best = -1, best_sad = 0; int bdx = 0, bdy = 0;
                 for (int c = 0; c < nc; ++c) {          /* spiral order, strict < */
                     int dx = cdx[c], dy = cdy[c];
                     long sad = 0;
@@ -168,17 +184,26 @@ int oracle_me(const uint8_t *cf, const uint8_t *const *rfs, int W, int H,
                             int b = ref_px(rf, W, H, x0 + ii + dx, y0 + j + dy);
                             sad += a > b ? a - b : b - a;
                         }
-                    if (best < 0 || sad < best) { best = sad; bdx = dx; bdy = dy; }
+                    long cost = sad + (long)lambda * se_bits(4 * dx) + (long)lambda * se_bits(4 * dy);
+                    if (best < 0 || cost < best) { best = cost; best_sad = sad; bdx = dx; bdy = dy; }
                 }
                 size_t o = ((size_t)i * n_rf + r) * 41 + p;
                 out_mvs[2 * o] = (int16_t)bdx; out_mvs[2 * o + 1] = (int16_t)bdy;
-                out_sads[o] = (uint16_t)best;
+                out_sads[o] = (uint16_t)best_sad;
             }
         }
     }
     free(cdx); free(cdy);
     (void)n_threads;
     return 0;
+}
+
+int oracle_me(const uint8_t *cf, const uint8_t *const *rfs, int W, int H,
+              int S, int n_rf, int sa_inclusive,
+              const int32_t *mb_list, int n_mb,
+              int16_t *out_mvs, uint16_t *out_sads, int n_threads)
+{
+    return oracle_me_rd(cf, rfs, W, H, S, n_rf, sa_inclusive, 0, mb_list, n_mb, out_mvs, out_sads, n_threads);
 }
 
 /* ------------------------------------------------------------------ O2 --
@@ -317,9 +342,9 @@ static long sad_q(const uint8_t *cf, const uint8_t *rf, int W, int H,
     return sad;
 }
 
-int oracle_sme(const uint8_t *cf, const uint8_t *const *rfs, int W, int H, int n_rf,
-               const int32_t *mb_list, int n_mb, const int16_t *in_mvs,
-               int16_t *out_qmvs, uint16_t *out_sads, int n_threads)
+int oracle_sme_rd(const uint8_t *cf, const uint8_t *const *rfs, int W, int H, int n_rf, int lambda,
+                  const int32_t *mb_list, int n_mb, const int16_t *in_mvs,
+                  int16_t *out_qmvs, uint16_t *out_sads, int n_threads)
 {
     if (W <= 0 || H <= 0 || n_rf < 1) return -1;
     int mb_cols = (W + 15) / 16;
@@ -336,24 +361,108 @@ int oracle_sme(const uint8_t *cf, const uint8_t *const *rfs, int W, int H, int n
                 int x0 = 16 * mbx + ox, y0 = 16 * mby + oy;
                 size_t o = ((size_t)i * n_rf + r) * 41 + p;
                 int cx = 4 * in_mvs[2 * o], cy = 4 * in_mvs[2 * o + 1];
-                long best = sad_q(cf, rfs[r], W, H, x0, y0, w, h, cx, cy);
+                /* cost J = SADq + lambda * R(v) (G18; lambda = 0: pure SAD, G13) */
+                long bsad = sad_q(cf, rfs[r], W, H, x0, y0, w, h, cx, cy);
+                long best = bsad + (long)lambda * (se_bits(cx) + se_bits(cy));
                 int bx = cx, by = cy;
                 for (int k = 0; k < 8; ++k) {                     /* half-pel ring */
                     int vx = cx + 2 * ring1[k][0], vy = cy + 2 * ring1[k][1];
                     long s = sad_q(cf, rfs[r], W, H, x0, y0, w, h, vx, vy);
-                    if (s < best) { best = s; bx = vx; by = vy; }
+                    long j = s + (long)lambda * (se_bits(vx) + se_bits(vy));
+                    if (j < best) { best = j; bsad = s; bx = vx; by = vy; }
                 }
                 int qx = bx, qy = by;
                 for (int k = 0; k < 8; ++k) {                     /* quarter-pel ring */
                     int vx = qx + ring1[k][0], vy = qy + ring1[k][1];
                     long s = sad_q(cf, rfs[r], W, H, x0, y0, w, h, vx, vy);
-                    if (s < best) { best = s; bx = vx; by = vy; }
+                    long j = s + (long)lambda * (se_bits(vx) + se_bits(vy));
+                    if (j < best) { best = j; bsad = s; bx = vx; by = vy; }
                 }
                 out_qmvs[2 * o] = (int16_t)bx; out_qmvs[2 * o + 1] = (int16_t)by;
-                out_sads[o] = (uint16_t)best;
+                out_sads[o] = (uint16_t)bsad;
             }
     }
     (void)n_threads;
+    return 0;
+}
+
+int oracle_sme(const uint8_t *cf, const uint8_t *const *rfs, int W, int H, int n_rf,
+               const int32_t *mb_list, int n_mb, const int16_t *in_mvs,
+               int16_t *out_qmvs, uint16_t *out_sads, int n_threads)
+{
+    return oracle_sme_rd(cf, rfs, W, H, n_rf, 0, mb_list, n_mb, in_mvs, out_qmvs, out_sads, n_threads);
+}
+
+/* ------------------------------------------------------------------ O4 --
+ * Mode decision ("According to the adopted distortion
+ * metric and the refined MVs from the SME, the best MB-partitioning mode is
+ * selected for each MB").  Per partition and RF: J_p(r) = SAD_p(r) +
+ * lambda * R(qmv_p(r)) (G18, from the SME outputs).  H.264 structure (G19):
+ *   mb_type 0 16x16: min_r J_0(r)
+ *           1 16x8 : sum over p in {1,2} of min_r J_p(r)
+ *           2 8x16 : sum over p in {3,4} of min_r J_p(r)
+ *           3 P8x8 : sum over sub-MBs s of min over sub_type t in {8x8, 8x4, 4x8,
+ *                    4x4} and r of sum over the sub-partitions of J_p(r)
+ *                    (one RF per 8x8: sub-8x8 partitions share it)
+ * Strict < everywhere, iterating mode, then sub_type, then r in increasing
+ * order (lowest index wins ties).  With lambda = 0 the P8x8/4x4 choice never
+ * loses (pin P4), so the decision is only informative with a rate term.
+ * out[n_mb][10]: mb_type, sub_type[4] (-1 unless P8x8), ref per 8x8 quadrant [4], cost. */
+int oracle_mode_decision(const int16_t *qmvs, const uint16_t *sads, int n_mb, int n_rf, int lambda,
+                         int32_t *out)
+{
+    if (n_mb < 0 || n_rf < 1 || n_rf > 16) return -1;
+    for (int i = 0; i < n_mb; ++i) {
+        long J[16][41];
+        for (int r = 0; r < n_rf; ++r)
+            for (int p = 0; p < 41; ++p) {
+                size_t o = ((size_t)i * n_rf + r) * 41 + p;
+                J[r][p] = (long)sads[o] + (long)lambda * (se_bits(qmvs[2 * o]) + se_bits(qmvs[2 * o + 1]));
+            }
+        long best = -1; int bt = 0, st[4] = {-1, -1, -1, -1}, rq[4] = {0, 0, 0, 0};
+        /* 16x16 */
+        { long c = -1; int cr = 0;
+          for (int r = 0; r < n_rf; ++r) if (c < 0 || J[r][0] < c) { c = J[r][0]; cr = r; }
+          best = c; bt = 0; for (int q = 0; q < 4; ++q) rq[q] = cr; }
+        /* 16x8 and 8x16 */
+        for (int t = 1; t <= 2; ++t) {
+            long c = 0; int pr[2];
+            for (int k = 0; k < 2; ++k) {
+                int p = (t == 1 ? 1 : 3) + k;
+                long m = -1;
+                for (int r = 0; r < n_rf; ++r) if (m < 0 || J[r][p] < m) { m = J[r][p]; pr[k] = r; }
+                c += m;
+            }
+            if (c < best) {
+                best = c; bt = t;
+                if (t == 1) { rq[0] = rq[1] = pr[0]; rq[2] = rq[3] = pr[1]; }
+                else        { rq[0] = rq[2] = pr[0]; rq[1] = rq[3] = pr[1]; }
+            }
+        }
+        /* P8x8 */
+        { long c = 0; int sst[4], srq[4];
+          for (int s = 0; s < 4; ++s) {
+              long m = -1;
+              for (int t = 0; t < 4; ++t)
+                  for (int r = 0; r < n_rf; ++r) {
+                      long v;
+                      if (t == 0) v = J[r][5 + s];
+                      else if (t == 1) v = J[r][9 + 2 * s] + J[r][10 + 2 * s];
+                      else if (t == 2) v = J[r][17 + 2 * s] + J[r][18 + 2 * s];
+                      else v = J[r][25 + 4 * s] + J[r][26 + 4 * s] + J[r][27 + 4 * s] + J[r][28 + 4 * s];
+                      if (m < 0 || v < m) { m = v; sst[s] = t; srq[s] = r; }
+                  }
+              c += m;
+          }
+          if (c < best) {
+              best = c; bt = 3;
+              for (int q = 0; q < 4; ++q) { st[q] = sst[q]; rq[q] = srq[q]; }
+          } }
+        int32_t *d = out + (size_t)i * 10;
+        d[0] = bt;
+        for (int q = 0; q < 4; ++q) { d[1 + q] = st[q]; d[5 + q] = rq[q]; }
+        d[9] = (int32_t)best;
+    }
     return 0;
 }
 

@@ -157,3 +157,70 @@ def sme(cf, rfs, mvs, S):
                 qmvs[o, r, p] = bv
                 sads[o, r, p] = best
     return qmvs, sads
+
+
+# ---------------------------------------------------- G18 rate term / O4 mode decision --
+
+def se_bits(v):
+    v = int(v)
+    k = 2 * v - 1 if v > 0 else -2 * v
+    return 2 * (k + 1).bit_length() - 1          # 2*floor(log2(k+1)) + 1
+
+
+def me_rd(cf, rfs, S, lam):
+    """brute force: lexicographic (SAD + lam*R(4mv), rank) minimum per partition"""
+    H, W = cf.shape
+    R = S // 2
+    mbc, mbr = -(-W // 16), -(-H // 16)
+    Wp, Hp = 16 * mbc, 16 * mbr
+    cfp = _edge(cf, ((0, Hp - H), (0, Wp - W)))
+    m = R + 1
+    d = np.arange(-R, R)
+    DX, DY = np.meshgrid(d, d)
+    rank = rank_closed_form(DX, DY).ravel()
+    rate = np.array([lam * (se_bits(4 * x) + se_bits(4 * y)) for x, y in zip(DX.ravel(), DY.ravel())])
+    parts = partitions()
+    mvs = np.zeros((mbr * mbc, len(rfs), 41, 2), np.int16)
+    sads = np.zeros((mbr * mbc, len(rfs), 41), np.uint16)
+    for r, rf in enumerate(rfs):
+        rfp = _edge(rf, ((m, m + Hp - H), (m, m + Wp - W)))
+        for o in range(mbr * mbc):
+            mby, mbx = divmod(o, mbc)
+            for p, (ox, oy, w, h) in enumerate(parts):
+                x0, y0 = 16 * mbx + ox, 16 * mby + oy
+                blk = cfp[y0:y0 + h, x0:x0 + w]
+                cand = np.array([np.abs(blk - rfp[y0 + dy + m:y0 + dy + m + h, x0 + dx + m:x0 + dx + m + w]).sum()
+                                 for dy, dx in zip(DY.ravel(), DX.ravel())])
+                best = np.lexsort((rank, cand + rate))[0]
+                mvs[o, r, p] = (DX.ravel()[best], DY.ravel()[best])
+                sads[o, r, p] = cand[best]
+    return mvs, sads
+
+
+def mode_decision(qmvs, sads, lam):
+    """enumerates every H.264 P-MB configuration (mb_type; per 8x8: sub_type, ref) explicitly"""
+    import itertools
+    n, n_rf = sads.shape[:2]
+    J = sads.astype(np.int64) + lam * np.vectorize(se_bits)(qmvs[..., 0]) + lam * np.vectorize(se_bits)(qmvs[..., 1])
+    sub_parts = {0: lambda s: [5 + s], 1: lambda s: [9 + 2 * s, 10 + 2 * s],
+                 2: lambda s: [17 + 2 * s, 18 + 2 * s], 3: lambda s: [25 + 4 * s + k for k in range(4)]}
+    out = np.zeros((n, 10), np.int32)
+    for i in range(n):
+        cands = []        # (cost, order key, result)
+        for r in range(n_rf):
+            cands.append((J[i, r, 0], (0, r), [0, -1, -1, -1, -1, r, r, r, r]))
+        for r1, r2 in itertools.product(range(n_rf), repeat=2):
+            cands.append((J[i, r1, 1] + J[i, r2, 2], (1, r1, r2), [1, -1, -1, -1, -1, r1, r1, r2, r2]))
+            cands.append((J[i, r1, 3] + J[i, r2, 4], (2, r1, r2), [2, -1, -1, -1, -1, r1, r2, r1, r2]))
+        per_s = []
+        for s in range(4):
+            opts = [(sum(J[i, r, p] for p in sub_parts[t](s)), (t, r)) for t in range(4) for r in range(n_rf)]
+            per_s.append(opts)
+        for combo in itertools.product(*per_s):
+            cost = sum(c for c, _ in combo)
+            key = (3,) + tuple(x for _, tr in combo for x in tr)
+            cands.append((cost, key, [3] + [tr[0] for _, tr in combo] + [tr[1] for _, tr in combo]))
+        cost, key, res = min(cands, key=lambda c: (c[0], c[1]))
+        out[i, :9] = res
+        out[i, 9] = cost
+    return out
