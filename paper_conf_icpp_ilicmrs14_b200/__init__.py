@@ -60,9 +60,10 @@ def lib():
         L.me_get_timings.argtypes = [P, P, P, P]
         L.me_set_fused.argtypes = [P, i]
         L.me_set_option.argtypes = [P, i, i]
+        L.me_mode_decision.argtypes = [P, P, P, P]
         for fn in ("me_set_stream", "me_set_rows", "me_get_layout", "me_estimate", "int_interpolate",
                    "sme_refine", "me_encode_frame", "me_last_launch_count", "me_stream_reset",
-                   "me_stream_push", "me_stream_outputs", "me_sync", "me_set_timing", "me_get_timings", "me_set_fused", "me_set_option"):
+                   "me_stream_push", "me_stream_outputs", "me_sync", "me_set_timing", "me_get_timings", "me_set_fused", "me_set_option", "me_mode_decision"):
             getattr(L, fn).restype = i
         _lib = L
     return _lib
@@ -212,7 +213,20 @@ class MotionEstimator:
         """SME fused into the ME kernel (default) or as its own launch."""
         _check(lib().me_set_fused(self._ctx, int(on)))
 
-    OPT_FUSED_SME, OPT_PIPELINE_RF, OPT_ME_CTAS_PER_SM = 1, 2, 3
+    OPT_FUSED_SME, OPT_PIPELINE_RF, OPT_ME_CTAS_PER_SM, OPT_LAMBDA = 1, 2, 3, 4
+
+    def set_lambda(self, lam: int):
+        """Rate term (f4, G18): ME and SME minimise SAD + lam * R(mv)."""
+        self.set_option(self.OPT_LAMBDA, lam)
+
+    def mode_decision(self, qmvs, qsads, out=None):
+        """Best H.264 P-MB configuration per MB (f2, me_mode_decision):
+        int32 [rows, mb_cols, 10] = mb_type, sub_type x4, ref per 8x8 x4, cost."""
+        o = out if out is not None else torch.empty((self.row1 - self.row0, self.mb_cols, 10), dtype=torch.int32,
+                                                    device=self.device)
+        self._bind_stream()
+        _check(lib().me_mode_decision(self._ctx, qmvs.data_ptr(), qsads.data_ptr(), o.data_ptr()))
+        return o
 
     def set_option(self, option: int, value: int):
         """me_set_option: scheduling knobs (results identical under every setting)."""

@@ -14,6 +14,7 @@
 
 #include "int_subpel.cuh"
 #include "me_fsbm.cuh"
+#include "mode_decision.cuh"
 #include "sme_refine.cuh"
 
 using namespace feves;
@@ -59,6 +60,9 @@ struct me_ctx {
   size_t me_smem_fused;
   int pipeline;          // per-RF ME launches, SME of RF k co-running with ME of RF k+1 (ME_OPT_PIPELINE_RF)
   int me_ctas_per_sm;    // cap on resident ME CTAs per SM (0 = hardware maximum; ME_OPT_ME_CTAS_PER_SM)
+  int lambda;            // G18 rate term (ME_OPT_LAMBDA); key = J * kmul + rank
+  uint32_t kmul;
+  int kshift;
   cudaStream_t sme_st;   // pipeline: SME stream
   cudaEvent_t ev_me[kMaxRf], ev_sme_done;
   int sf_v0[kMaxRf], sf_v1[kMaxRf];   // MB rows whose SF rows each SF-ring slot holds (re-split support)
@@ -92,7 +96,9 @@ static cudaError_t set_me_smem(int bytes) {
   cudaError_t e = cudaSuccess;
   for (auto fn : {me_fsbm_kernel<0>, me_fsbm_kernel<16>, me_fsbm_kernel<32>, me_fsbm_kernel<64>, me_fsbm_kernel<128>,
                   me_fsbm_kernel<0, true>, me_fsbm_kernel<16, true>, me_fsbm_kernel<32, true>,
-                  me_fsbm_kernel<64, true>, me_fsbm_kernel<128, true>})
+                  me_fsbm_kernel<64, true>, me_fsbm_kernel<128, true>,
+                  me_fsbm_kernel<0, false, 15>, me_fsbm_kernel<16, false, 15>, me_fsbm_kernel<32, false, 15>,
+                  me_fsbm_kernel<64, false, 15>, me_fsbm_kernel<128, false, 15>})
     if (e == cudaSuccess) e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
   return e;
 }
@@ -101,6 +107,22 @@ static int launch_status() {
   const cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) { fprintf(stderr, "feves_me: %s\n", cudaGetErrorString(e)); return ME_ECUDA; }
   return ME_OK;
+}
+
+// key addend table E[dy+R][dx+R] = lambda * R(4dx, 4dy) * kmul + spiral rank (G4, G18):
+// with lambda = 0 this is the spiral rank and key = SAD * 2^16 + rank; with a rate
+// term J = SAD + lambda*R may exceed 16 bits, so key = J * 2^15 + rank (rank < 2^15
+// for S <= 128, J < 2^17 for lambda <= 2000).
+static int upload_key_table(me_ctx* c) {
+  const int S = c->S;
+  c->kshift = c->lambda ? 15 : 16;
+  c->kmul = 1u << c->kshift;
+  std::vector<uint32_t> e((size_t)S * S);
+  for (int dy = -c->R; dy < c->R; ++dy)
+    for (int dx = -c->R; dx < c->R; ++dx)
+      e[(size_t)(dy + c->R) * S + (dx + c->R)] =
+          (uint32_t)(c->lambda * (se_bits(4 * dx) + se_bits(4 * dy))) * c->kmul + (uint32_t)spiral_rank_closed_form(dx, dy);
+  return cudaMemcpy(c->d_rank, e.data(), e.size() * 4, cudaMemcpyHostToDevice) == cudaSuccess ? ME_OK : ME_ECUDA;
 }
 
 // ------------------------------------------------------------ lifetime ----
@@ -129,22 +151,19 @@ extern "C" me_ctx* me_create(int width, int height, int sa_range, int n_rf) {
   c->pipeline = 0;
   c->me_ctas_per_sm = 0;
 
-  std::vector<uint32_t> rank((size_t)S * S), inv((size_t)(S + 1) * (S + 1), 0);
+  std::vector<uint32_t> inv((size_t)(S + 1) * (S + 1), 0);
   for (int dy = -c->R; dy < c->R; ++dy)
-    for (int dx = -c->R; dx < c->R; ++dx) {
-      const int r = spiral_rank_closed_form(dx, dy);
-      rank[(size_t)(dy + c->R) * S + (dx + c->R)] = (uint32_t)r;
-      inv[r] = (uint32_t)(uint16_t)dx | ((uint32_t)(uint16_t)dy << 16);
-    }
+    for (int dx = -c->R; dx < c->R; ++dx)
+      inv[spiral_rank_closed_form(dx, dy)] = (uint32_t)(uint16_t)dx | ((uint32_t)(uint16_t)dy << 16);
   const size_t nmv = (size_t)c->mb_cols * c->mb_rows * n_rf * kNPart;
-  bool ok = cudaMalloc(&c->d_rank, rank.size() * 4) == cudaSuccess &&
+  bool ok = cudaMalloc(&c->d_rank, (size_t)S * S * 4) == cudaSuccess &&
             cudaMalloc(&c->d_inv, inv.size() * 4) == cudaSuccess &&
             cudaMalloc(&c->d_mvs, nmv * 4) == cudaSuccess &&
             cudaMalloc(&c->d_sads, nmv * 2) == cudaSuccess &&
             cudaStreamCreateWithFlags(&c->stream, cudaStreamNonBlocking) == cudaSuccess;
   if (ok) {
     c->own_stream = true;
-    ok = cudaMemcpy(c->d_rank, rank.data(), rank.size() * 4, cudaMemcpyHostToDevice) == cudaSuccess &&
+    ok = upload_key_table(c) == ME_OK &&
          cudaMemcpy(c->d_inv, inv.data(), inv.size() * 4, cudaMemcpyHostToDevice) == cudaSuccess &&
          set_me_smem(200 * 1024) == cudaSuccess;   // max; the launch asks for what it needs
   }
@@ -251,6 +270,7 @@ static int launch_me(me_ctx* c, const uint8_t* cf, const uint8_t* const* rfs, in
   P.W = c->W; P.H = c->H; P.S = c->S; P.R = c->R; P.n_rf = n_ref; P.rf_stride = c->n_rf;
   P.mb_cols = c->mb_cols; P.row0 = c->row0;
   P.rank_tab = c->d_rank; P.inv_tab = c->d_inv;
+  P.kmul = c->kmul; P.kshift = c->kshift; P.lambda = c->lambda;
   P.out_mvs = mvs; P.out_sads = sads;
   bool vec = (c->W % 16 == 0) && (c->R % 16 == 0);
   for (int k = 0; k < n_ref; ++k) vec = vec && ((reinterpret_cast<uintptr_t>(rfs[k]) & 15) == 0);
@@ -271,6 +291,7 @@ static int launch_me(me_ctx* c, const uint8_t* cf, const uint8_t* const* rfs, in
 #define FEVES_ME_LAUNCH(SS)                                                              \
   do {                                                                                   \
     if (fused) me_fsbm_kernel<SS, true><<<grid, c->me_threads, smem, st>>>(P);          \
+    else if (c->lambda) me_fsbm_kernel<SS, false, 15><<<grid, c->me_threads, smem, st>>>(P); \
     else me_fsbm_kernel<SS, false><<<grid, c->me_threads, smem, st>>>(P);               \
   } while (0)
   switch (c->S) {   // compile-time window geometry for the paper's SA sizes (Fig. 6a: 32..256)
@@ -332,11 +353,13 @@ static int launch_sme(me_ctx* c, const uint8_t* cf, const uint8_t* const* sfs, c
   P.W = c->W; P.H = c->H; P.n_rf = n_ref; P.rf_stride = c->n_rf; P.mb_cols = c->mb_cols; P.row0 = c->row0;
   P.n_rows = c->row1 - c->row0;
   P.groups = (c->mb_cols + 7) / 8;
+  P.lambda = c->lambda;
   P.pad = c->sf_pad; P.pitch = c->sf_pitch;
   P.plane = (size_t)c->sf_rows * c->sf_pitch;
   const int warps = n_ref * P.n_rows * P.groups;
   tmark(c, 4, st);
-  sme_refine_kernel<<<dim3((warps + 3) / 4, 7), 128, 0, st>>>(P);   // y = partition mode
+  if (c->lambda) sme_refine_kernel<true><<<dim3((warps + 3) / 4, 7), 128, 0, st>>>(P);   // y = partition mode
+  else sme_refine_kernel<false><<<dim3((warps + 3) / 4, 7), 128, 0, st>>>(P);
   tmark(c, 5, st);
   c->last_launches++;
   return launch_status();
@@ -429,7 +452,7 @@ extern "C" int me_encode_frame(me_ctx* c, const uint8_t* cf, const uint8_t* cons
   int st;
   for (int k = 0; k < n_int; ++k)
     if ((st = launch_int(c, rfs[k], sfs[k], c->stream)) != ME_OK) return st;
-  if (c->fuse)   // ME with the SME fused into the same CTAs (one launch)
+  if (c->fuse && !c->lambda)   // ME with the SME fused into the same CTAs (one launch; pure SAD only)
     return launch_me(c, cf, rfs, out_mvs, out_sads, c->n_rf, c->stream, reinterpret_cast<const uint8_t* const*>(sfs),
                      out_qmvs, out_qsads);
   return run_me_sme(c, cf, rfs, reinterpret_cast<const uint8_t* const*>(sfs), mvs, sads, out_qmvs, out_qsads, c->n_rf,
@@ -535,7 +558,7 @@ extern "C" int me_stream_push(me_ctx* c, const uint8_t* cf, int cf_on_host, int1
     uint16_t* qs = (out_qsads && !out_on_host) ? out_qsads : (out_on_host ? c->d_qsads2[par] : c->d_qsads);
     // the device output buffer t & 1 is free once the download of push t-2 finished
     if (out_on_host && cudaStreamWaitEvent(c->stream, c->ev_down[par], 0) != cudaSuccess) return launch_status();
-    if (c->fuse) {
+    if (c->fuse && !c->lambda) {
       // fused: the SME of ref 0 reads SF(t-1), so INT(t-1) runs first on the same stream
       if ((st = launch_int(c, new_rf, new_sf, c->stream)) != ME_OK) return st;
       if ((st = launch_me(c, cur, rfs, nullptr, nullptr, n_ref, c->stream, sfs, qm, qs)) != ME_OK) return st;
@@ -613,8 +636,28 @@ extern "C" int me_set_option(me_ctx* c, int option, int value) {
       if (value < 0 || value > 32) return ME_EINVAL;
       c->me_ctas_per_sm = value;
       return ME_OK;
+    case ME_OPT_LAMBDA:
+      if (value < 0 || value > 2000) return ME_EINVAL;
+      if (c->stream) cudaStreamSynchronize(c->stream);   // the table may be in use
+      c->lambda = value;
+      return upload_key_table(c);
     default: return ME_EINVAL;
   }
 }
 
 extern "C" int me_set_fused(me_ctx* c, int on) { return me_set_option(c, ME_OPT_FUSED_SME, on); }
+
+extern "C" int me_mode_decision(me_ctx* c, const int16_t* qmvs, const uint16_t* qsads, int32_t* out_modes) {
+  if (!c || !is_device_ptr(c, qmvs) || !is_device_ptr(c, qsads) || !is_device_ptr(c, out_modes)) return ME_EINVAL;
+  ModeParams P;
+  P.qmvs = reinterpret_cast<const uint32_t*>(qmvs);
+  P.sads = qsads;
+  P.out = out_modes;
+  P.n_mb = (c->row1 - c->row0) * c->mb_cols;
+  P.n_rf = c->n_rf;
+  P.lambda = c->lambda;
+  c->last_launches = 0;
+  mode_decision_kernel<<<(P.n_mb + 127) / 128, 128, 0, c->stream>>>(P);
+  c->last_launches++;
+  return launch_status();
+}

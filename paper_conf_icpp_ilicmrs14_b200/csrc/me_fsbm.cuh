@@ -37,8 +37,10 @@ struct MeParams {
   int W, H, S, R, n_rf;       // n_rf = RFs searched by this launch (RF ramp)
   int rf_stride;              // RF dimension of the output layout (the context's n_rf)
   int mb_cols, row0;
-  const uint32_t* rank_tab;   // [S][S], [dy+R][dx+R] -> spiral rank (G4)
+  const uint32_t* rank_tab;   // [S][S], [dy+R][dx+R] -> key addend E = lambda*R(4dx,4dy)*kmul + spiral rank (G4, G18)
   const uint32_t* inv_tab;    // rank -> (dx & 0xffff) | (dy << 16)
+  uint32_t kmul;              // key = J * kmul + rank: 2^16 (lambda = 0) or 2^15 (J may exceed 16 bits)
+  int kshift, lambda;
   int16_t* out_mvs;
   uint16_t* out_sads;
   int vec_ok;                 // 16-byte aligned rows and window start: vector staging allowed
@@ -77,12 +79,25 @@ constexpr uint32_t kSh = 65536u;
 // Keys of every partition completed by 4x4 block row BY of one candidate.
 // L = the four 4x4 SADs of this block row; key = SAD * 2^16 + rank.  Every key
 // is ONE IMAD (FMA pipe) on a child's SAD or key; plain sums are IMAD.IADD.
-// key(parent) = sad(other child) * 2^16 + key(child): one IMAD.  Written as
-// inline PTX so the compiler cannot re-associate it into add-then-IMAD.
+// key(parent) = sad(other child) * 2^KSH + key(child): one IMAD with an immediate.
+// Written as inline PTX so the compiler cannot re-associate it into add-then-IMAD.
+template <int KSH>
 __device__ __forceinline__ uint32_t kmad(uint32_t sad, uint32_t key) {
   uint32_t d;
-  asm("mad.lo.u32 %0, %1, 65536, %2;" : "=r"(d) : "r"(sad), "r"(key));
+  asm("mad.lo.u32 %0, %1, %2, %3;" : "=r"(d) : "r"(sad), "n"(1 << KSH), "r"(key));
   return d;
+}
+
+// G18: Exp-Golomb se(v) bit length, R(mv) = se(mv.x) + se(mv.y) (quarter-pel)
+__host__ __device__ __forceinline__ int se_bits(int v) {
+  const unsigned k = v > 0 ? 2u * (unsigned)v - 1u : 2u * (unsigned)(-v);
+#ifdef __CUDA_ARCH__
+  return 2 * (31 - __clz((int)(k + 1u))) + 1;
+#else
+  int n = 0;
+  while ((k + 1u) >> (n + 1)) ++n;
+  return 2 * n + 1;
+#endif
 }
 
 // plain SAD sum kept on the FMA pipe: the ALU pipe is the bottleneck, and an
@@ -94,16 +109,16 @@ __device__ __forceinline__ uint32_t fadd(uint32_t a, uint32_t b, uint32_t one) {
   return d;
 }
 
-template <int BY>
+template <int BY, int KSH>
 __device__ __forceinline__ void block_row_keys(const uint32_t (&L)[4], uint32_t rank, RowState& st,
                                                uint32_t (&K)[16], uint32_t one) {
   uint32_t k4[4];
 #pragma unroll
-  for (int i = 0; i < 4; ++i) k4[i] = kmad(L[i], rank);                   // 4x4
+  for (int i = 0; i < 4; ++i) k4[i] = kmad<KSH>(L[i], rank);                   // 4x4
 #pragma unroll
   for (int i = 0; i < 4; ++i) K[i] = k4[i];
-  K[4] = kmad(L[1], k4[0]);                                                // 8x4
-  K[5] = kmad(L[3], k4[2]);
+  K[4] = kmad<KSH>(L[1], k4[0]);                                                // 8x4
+  K[5] = kmad<KSH>(L[3], k4[2]);
   const uint32_t p84_0 = fadd(L[0], L[1], one), p84_1 = fadd(L[2], L[3], one);
   if ((BY & 1) == 0) {
 #pragma unroll
@@ -111,20 +126,20 @@ __device__ __forceinline__ void block_row_keys(const uint32_t (&L)[4], uint32_t 
     st.p84top[0] = p84_0; st.p84top[1] = p84_1;
   } else {
 #pragma unroll
-    for (int i = 0; i < 4; ++i) K[6 + i] = kmad(L[i], st.k4prev[i]);      // 4x8
+    for (int i = 0; i < 4; ++i) K[6 + i] = kmad<KSH>(L[i], st.k4prev[i]);      // 4x8
     const uint32_t p88_0 = fadd(p84_0, st.p84top[0], one), p88_1 = fadd(p84_1, st.p84top[1], one);
-    const uint32_t k88_0 = kmad(p88_0, rank), k88_1 = kmad(p88_1, rank);  // 8x8
+    const uint32_t k88_0 = kmad<KSH>(p88_0, rank), k88_1 = kmad<KSH>(p88_1, rank);  // 8x8
     K[10] = k88_0;
     K[11] = k88_1;
-    const uint32_t k168 = kmad(p88_1, k88_0);                              // 16x8
+    const uint32_t k168 = kmad<KSH>(p88_1, k88_0);                              // 16x8
     K[12] = k168;
     if (BY == 1) {
       st.p88top[0] = p88_0; st.p88top[1] = p88_1;
       st.p168top = fadd(p88_0, p88_1, one);
     } else {
-      K[13] = kmad(st.p88top[0], k88_0);                                    // 8x16 left
-      K[14] = kmad(st.p88top[1], k88_1);                                    // 8x16 right
-      K[15] = kmad(st.p168top, k168);                                       // 16x16
+      K[13] = kmad<KSH>(st.p88top[0], k88_0);                                    // 8x16 left
+      K[14] = kmad<KSH>(st.p88top[1], k88_1);                                    // 8x16 right
+      K[15] = kmad<KSH>(st.p168top, k168);                                       // 16x16
     }
   }
 }
@@ -257,8 +272,9 @@ __device__ __forceinline__ void fused_sme(const MeParams& P, const uint32_t* cf_
 }
 
 // S_CT = compile-time SA size (0 = any even S read from P at run time);
-// FUSE = also run the SME of this MB (fused_sme) after its ME.
-template <int S_CT, bool FUSE = false>
+// FUSE = also run the SME of this MB (fused_sme) after its ME;
+// KSH = key shift: 16 (pure SAD) or 15 (rate term, G18: J may exceed 16 bits).
+template <int S_CT, bool FUSE = false, int KSH = 16>
 __global__ void __launch_bounds__(128, 4) me_fsbm_kernel(const MeParams P) {
   extern __shared__ __align__(16) uint32_t smem[];
   const int S = S_CT ? S_CT : P.S;
@@ -370,10 +386,10 @@ __global__ void __launch_bounds__(128, 4) me_fsbm_kernel(const MeParams P) {
             for (int b = 0; b < 4; ++b) acc[t][b] = vad4(cw[b], w[b], (r & 3) ? acc[t][b] : 0u);
             if ((r & 3) == 3) {
               const int by = r >> 2;
-              if (by == 0) block_row_keys<0>(acc[t], rank[t], st[t], Kp[t], one);
-              if (by == 1) block_row_keys<1>(acc[t], rank[t], st[t], Kp[t], one);
-              if (by == 2) block_row_keys<2>(acc[t], rank[t], st[t], Kp[t], one);
-              if (by == 3) block_row_keys<3>(acc[t], rank[t], st[t], Kp[t], one);
+              if (by == 0) block_row_keys<0, KSH>(acc[t], rank[t], st[t], Kp[t], one);
+              if (by == 1) block_row_keys<1, KSH>(acc[t], rank[t], st[t], Kp[t], one);
+              if (by == 2) block_row_keys<2, KSH>(acc[t], rank[t], st[t], Kp[t], one);
+              if (by == 3) block_row_keys<3, KSH>(acc[t], rank[t], st[t], Kp[t], one);
               if (t & 1) {                                  // pair (t-1, t) finished this block row
                 if (by == 0) fold_pair<0>(M, Kp[t - 1], Kp[t]);
                 if (by == 1) fold_pair<1>(M, Kp[t - 1], Kp[t]);
@@ -396,15 +412,18 @@ __global__ void __launch_bounds__(128, 4) me_fsbm_kernel(const MeParams P) {
     for (int p = threadIdx.x; p < kNPart; p += blockDim.x) {
       uint32_t k = red[p];
       for (int w = 1; w < nwarps; ++w) k = min(k, red[w * kNPart + p]);
-      const uint32_t mv = __ldg(P.inv_tab + (k & 0xffffu));
+      const uint32_t mv = __ldg(P.inv_tab + (k & ((1u << KSH) - 1u)));
+      uint32_t sad = k >> KSH;                               // J = SAD + lambda*R(mv) (G18)
+      if (KSH != 16)
+        sad -= (uint32_t)(P.lambda * (se_bits(4 * (int)(int16_t)(mv & 0xffffu)) + se_bits(4 * (int)(int16_t)(mv >> 16))));
       const size_t o = ((size_t)(blockIdx.y * P.mb_cols + mbx) * P.rf_stride + ref) * kNPart + p;
       if (P.out_mvs) {
         reinterpret_cast<uint32_t*>(P.out_mvs)[o] = mv;
-        P.out_sads[o] = (uint16_t)(k >> 16);
+        P.out_sads[o] = (uint16_t)sad;
       }
       if (FUSE) {
         win_mv[ref * kNPart + p] = mv;
-        win_sad[ref * kNPart + p] = k >> 16;
+        win_sad[ref * kNPart + p] = sad;
       }
     }
   }

@@ -17,6 +17,7 @@
 // every lane of a partition then holds the same (best, bestv) -- no divergence.
 #pragma once
 #include "common.cuh"
+#include "me_fsbm.cuh"   // se_bits (G18)
 
 namespace feves {
 
@@ -31,6 +32,7 @@ struct SmeParams {
   int groups;                                         // ceil(mb_cols / 8)
   int pad, pitch;
   size_t plane;
+  int lambda;                                         // G18 rate term (0 = pure SAD, G13)
 };
 
 // ring-1 spiral order s_k (G12/G14), compile-time so unrolled loops fold it
@@ -90,7 +92,8 @@ __device__ __forceinline__ int mode_part(int bx, int by) {
 // Axis neighbour (dx,0) = avg(HP(0,0), HP(dx,0)), (0,dy) likewise; diagonal
 // (dx,dy) = avg of the two corners of the half-grid unit square that have one
 // odd coordinate: (0,0) & (dx,dy) if H has mixed parity, else (dx,0) & (0,dy).
-template <int MODE, int YG, int XMASK>
+// RD = rate term (G18) compiled in
+template <int MODE, int YG, int XMASK, bool RD>
 __device__ __forceinline__ void refine_mode(const SmeParams& P, const uint8_t* __restrict__ sf, size_t o, int bx,
                                             int xs, int ys0, bool writer, const uint32_t (&cfs)[16]) {
   constexpr int NG = 4 / YG;           // partitions (block groups) inside this lane's strip
@@ -112,6 +115,7 @@ __device__ __forceinline__ void refine_mode(const SmeParams& P, const uint8_t* _
                              cfs + 4 * (g * YG + j));
       best[g] = xsum<XMASK>(s);
     }
+    if (RD) best[g] += P.lambda * (se_bits(bvx[g]) + se_bits(bvy[g]));   // J at the centre
   }
   // ---- half stage (all 8 candidates' loads first: latency-bound) ----
   {
@@ -134,8 +138,10 @@ __device__ __forceinline__ void refine_mode(const SmeParams& P, const uint8_t* _
     for (int k = 0; k < 8; ++k)
 #pragma unroll
       for (int g = 0; g < NG; ++g) {
-        const uint32_t t = xsum<XMASK>(sad[k][g]);
-        if (t < best[g]) { best[g] = t; bvx[g] = ox[g] + 2 * c_ring1[k][0]; bvy[g] = oy[g] + 2 * c_ring1[k][1]; }
+        const int vx = ox[g] + 2 * c_ring1[k][0], vy = oy[g] + 2 * c_ring1[k][1];
+        uint32_t t = xsum<XMASK>(sad[k][g]);
+        if (RD) t += P.lambda * (se_bits(vx) + se_bits(vy));
+        if (t < best[g]) { best[g] = t; bvx[g] = vx; bvy[g] = vy; }
       }
   }
   // ---- quarter stage from the 3x3 half-grid windows around the best half position ----
@@ -181,8 +187,10 @@ __device__ __forceinline__ void refine_mode(const SmeParams& P, const uint8_t* _
     const int ox = bvx[g], oy = bvy[g];
 #pragma unroll
     for (int k = 0; k < 8; ++k) {             // spiral order, strict < (G14)
-      const uint32_t t = xsum<XMASK>(qs[k]);
-      if (t < best[g]) { best[g] = t; bvx[g] = ox + c_ring1[k][0]; bvy[g] = oy + c_ring1[k][1]; }
+      const int vx = ox + c_ring1[k][0], vy = oy + c_ring1[k][1];
+      uint32_t t = xsum<XMASK>(qs[k]);
+      if (RD) t += P.lambda * (se_bits(vx) + se_bits(vy));
+      if (t < best[g]) { best[g] = t; bvx[g] = vx; bvy[g] = vy; }
     }
   }
   if (writer && (bx & XMASK) == 0) {     // partition leader lane writes
@@ -190,11 +198,12 @@ __device__ __forceinline__ void refine_mode(const SmeParams& P, const uint8_t* _
     for (int g = 0; g < NG; ++g) {
       const int p = mode_part<MODE>(bx, g * YG);
       P.out_qmvs[o + p] = (uint32_t)(uint16_t)bvx[g] | ((uint32_t)(uint16_t)bvy[g] << 16);
-      P.out_sads[o + p] = (uint16_t)best[g];
+      P.out_sads[o + p] = (uint16_t)(best[g] - (RD ? P.lambda * (se_bits(bvx[g]) + se_bits(bvy[g])) : 0));
     }
   }
 }
 
+template <bool RD>
 __global__ void __launch_bounds__(128) sme_refine_kernel(const SmeParams P) {
   const int warp_id = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
   const int n_warps = P.n_rf * P.n_rows * P.groups;
@@ -215,13 +224,13 @@ __global__ void __launch_bounds__(128) sme_refine_kernel(const SmeParams P) {
   const uint8_t* __restrict__ sf = P.sf[ref];
   const size_t o = ((size_t)(mrow * P.mb_cols + mbx) * P.rf_stride + ref) * kNPart;
   switch (blockIdx.y) {   // one mode per warp: 7x the independent warps (the kernel is latency-bound)
-    case 0: refine_mode<0, 4, 3>(P, sf, o, bx, xs, ys0, writer, cfs); break;   // 16x16
-    case 1: refine_mode<1, 2, 3>(P, sf, o, bx, xs, ys0, writer, cfs); break;   // 16x8
-    case 2: refine_mode<2, 4, 1>(P, sf, o, bx, xs, ys0, writer, cfs); break;   // 8x16
-    case 3: refine_mode<3, 2, 1>(P, sf, o, bx, xs, ys0, writer, cfs); break;   // 8x8
-    case 4: refine_mode<4, 1, 1>(P, sf, o, bx, xs, ys0, writer, cfs); break;   // 8x4
-    case 5: refine_mode<5, 2, 0>(P, sf, o, bx, xs, ys0, writer, cfs); break;   // 4x8
-    default: refine_mode<6, 1, 0>(P, sf, o, bx, xs, ys0, writer, cfs); break;  // 4x4
+    case 0: refine_mode<0, 4, 3, RD>(P, sf, o, bx, xs, ys0, writer, cfs); break;   // 16x16
+    case 1: refine_mode<1, 2, 3, RD>(P, sf, o, bx, xs, ys0, writer, cfs); break;   // 16x8
+    case 2: refine_mode<2, 4, 1, RD>(P, sf, o, bx, xs, ys0, writer, cfs); break;   // 8x16
+    case 3: refine_mode<3, 2, 1, RD>(P, sf, o, bx, xs, ys0, writer, cfs); break;   // 8x8
+    case 4: refine_mode<4, 1, 1, RD>(P, sf, o, bx, xs, ys0, writer, cfs); break;   // 8x4
+    case 5: refine_mode<5, 2, 0, RD>(P, sf, o, bx, xs, ys0, writer, cfs); break;   // 4x8
+    default: refine_mode<6, 1, 0, RD>(P, sf, o, bx, xs, ys0, writer, cfs); break;  // 4x4
   }
 }
 

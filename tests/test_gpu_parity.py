@@ -323,3 +323,31 @@ def test_stream_host_pipeline_many_frames(feves, orc):
         np.testing.assert_array_equal(outs[t][0].numpy().reshape(n, n_rf, 41, 2), o_q)
         np.testing.assert_array_equal(outs[t][1].numpy().reshape(n, n_rf, 41), o_s)
     me.close()
+
+
+@pytest.mark.parametrize("lam,S", [(4, 16), (25, 32), (200, 8)])
+def test_rate_term_me_sme_and_mode_decision(feves, orc, lam, S):
+    """f4 (G18) and f2 (O4) on the GPU path vs the oracle, bit-exact"""
+    W, H, n_rf = 80, 48, 2
+    cf, rfs = _frames("tex", W, H, n_rf, 3 + lam)
+    me = feves.MotionEstimator(W, H, S, n_rf)
+    me.set_lambda(lam)
+    tcf, trfs = _dev(cf), [_dev(r) for r in rfs]
+    sfs = [me.new_sf() for _ in trfs]
+    (m, s), (q, qs) = me.encode_frame(tcf, trfs, sfs, n_int=n_rf, out_me=me.new_mvs())
+    modes = me.mode_decision(q, qs)
+    torch.cuda.synchronize()
+    n = me.mb_rows * me.mb_cols
+    o_m, o_s = orc.me(cf, rfs, S, lam=lam)
+    np.testing.assert_array_equal(m.cpu().numpy().reshape(n, n_rf, 41, 2), o_m)
+    np.testing.assert_array_equal(s.cpu().numpy().reshape(n, n_rf, 41), o_s)
+    o_q, o_qs = orc.sme(cf, rfs, o_m, lam=lam)
+    np.testing.assert_array_equal(q.cpu().numpy().reshape(n, n_rf, 41, 2), o_q)
+    np.testing.assert_array_equal(qs.cpu().numpy().reshape(n, n_rf, 41), o_qs)
+    np.testing.assert_array_equal(modes.cpu().numpy().reshape(n, 10), orc.mode_decision(o_q, o_qs, lam))
+    me.set_lambda(0)                                     # back to pure SAD: original results
+    (m0, s0), _ = me.encode_frame(tcf, trfs, sfs, n_int=0, out_me=me.new_mvs())
+    torch.cuda.synchronize()
+    o_m0, o_s0 = orc.me(cf, rfs, S)
+    np.testing.assert_array_equal(m0.cpu().numpy().reshape(n, n_rf, 41, 2), o_m0)
+    me.close()
