@@ -13,6 +13,7 @@ arithmetic step of the method lives in that C file, which cites the passage of
   me                 O1  (P:6)         P1 hand-computed, P2, P3, P4, P9 NumPy brute force
   me(lam>0), sme(lam>0)  G18 (f4)      P12 hand-computed rate pins, P13 NumPy brute force
   mode_decision      O4  (f2)    P14 closed forms, P13 NumPy enumeration
+  sme(satd=True)     G20 (f4)          P15 Hadamard closed forms, P13 NumPy (scipy Hadamard) SME
   sample/int_planes  O2  (P:6)  P5 closed forms + golden, P6, P7, P9
   sme                O3  (P:6)   P2, P8 (incl. half-pel synthetic), P9
 """
@@ -53,6 +54,9 @@ def lib():
         L.oracle_me_rd.argtypes = [P, P, i, i, i, i, i, i, P, i, P, P, i]
         L.oracle_sme.argtypes = [P, P, i, i, i, P, i, P, P, P, i]
         L.oracle_sme_rd.argtypes = [P, P, i, i, i, i, P, i, P, P, P, i]
+        L.oracle_sme_ex.argtypes = [P, P, i, i, i, i, i, P, i, P, P, P, i]
+        L.oracle_satd_q.argtypes = [P, P, i, i, i, i, i, i, i, i]
+        L.oracle_satd_q.restype = ctypes.c_long
         L.oracle_mode_decision.argtypes = [P, P, i, i, i, P]
         L.oracle_mv_bits.argtypes = [i, i]
         L.oracle_mv_bits.restype = i
@@ -120,9 +124,9 @@ def me(cf, rfs, sa_range: int, mb_list=None, sa_inclusive: bool = False, threads
     return mvs, sads
 
 
-def sme(cf, rfs, in_mvs, mb_list=None, threads: int = 0, lam: int = 0):
-    """O3 (lam > 0: cost J = SAD + lam * R(qmv), G18). in_mvs int16 [n_mb, n_rf, 41, 2]
-    full-pel. Returns (qmvs, sads)."""
+def sme(cf, rfs, in_mvs, mb_list=None, threads: int = 0, lam: int = 0, satd: bool = False):
+    """O3 (lam > 0: cost J = D + lam * R(qmv), G18; satd: D = Hadamard SATD, G20).
+    in_mvs int16 [n_mb, n_rf, 41, 2] full-pel. Returns (qmvs, distortions)."""
     cf = _u8(cf)
     rfs = [_u8(r) for r in rfs]
     H, W = cf.shape
@@ -131,11 +135,17 @@ def sme(cf, rfs, in_mvs, mb_list=None, threads: int = 0, lam: int = 0):
     in_mvs = np.ascontiguousarray(in_mvs, np.int16).reshape(n, len(rfs), N_PART, 2)
     qmvs = np.zeros((n, len(rfs), N_PART, 2), np.int16)
     sads = np.zeros((n, len(rfs), N_PART), np.uint16)
-    rc = lib().oracle_sme_rd(_ptr(cf), _ptr_array(rfs), W, H, len(rfs), int(lam), _ptr(mb_list), n,
+    rc = lib().oracle_sme_ex(_ptr(cf), _ptr_array(rfs), W, H, len(rfs), int(lam), int(satd), _ptr(mb_list), n,
                              _ptr(in_mvs), _ptr(qmvs), _ptr(sads), threads)
     if rc != 0:
         raise ValueError("oracle_sme: bad arguments")
     return qmvs, sads
+
+
+def satd_q(cf, rf, x0, y0, w, h, vx, vy) -> int:
+    """G20 SATD of the w x h block at (x0, y0) against rf at quarter-pel offset (vx, vy)."""
+    cf, rf = _u8(cf), _u8(rf)
+    return int(lib().oracle_satd_q(_ptr(cf), _ptr(rf), cf.shape[1], cf.shape[0], x0, y0, w, h, vx, vy))
 
 
 def mv_bits(qx: int, qy: int) -> int:

@@ -342,7 +342,60 @@ static long sad_q(const uint8_t *cf, const uint8_t *rf, int W, int H,
     return sad;
 }
 
+/* G20 (f4, JM "UseHadamard"): SATD of a partition = sum over its 4x4 blocks of
+ * (sum |H D H^T| + 1) >> 1, D = CF - prediction, H = the 4x4 Hadamard matrix.
+ * Written as the matrix products (no fast butterfly).                       */
+static const int H4[4][4] = { {1, 1, 1, 1}, {1, 1, -1, -1}, {1, -1, -1, 1}, {1, -1, 1, -1} };
+
+static long satd_q(const uint8_t *cf, const uint8_t *rf, int W, int H,
+                   int x0, int y0, int w, int h, int vx, int vy)
+{
+    long total = 0;
+    for (int by = 0; by < h; by += 4)
+        for (int bx = 0; bx < w; bx += 4) {
+            long D[4][4], T[4][4], U[4][4];
+            for (int j = 0; j < 4; ++j)
+                for (int i = 0; i < 4; ++i) {
+                    int X = x0 + bx + i, Y = y0 + by + j;
+                    D[j][i] = ref_px(cf, W, H, X, Y) - oracle_sample(rf, W, H, 4 * X + vx, 4 * Y + vy);
+                }
+            for (int a = 0; a < 4; ++a)            /* T = H D */
+                for (int b = 0; b < 4; ++b) {
+                    T[a][b] = 0;
+                    for (int k = 0; k < 4; ++k) T[a][b] += H4[a][k] * D[k][b];
+                }
+            for (int a = 0; a < 4; ++a)            /* U = T H^T */
+                for (int b = 0; b < 4; ++b) {
+                    U[a][b] = 0;
+                    for (int k = 0; k < 4; ++k) U[a][b] += T[a][k] * H4[b][k];
+                }
+            long sum = 0;
+            for (int a = 0; a < 4; ++a)
+                for (int b = 0; b < 4; ++b) sum += U[a][b] < 0 ? -U[a][b] : U[a][b];
+            total += (sum + 1) >> 1;
+        }
+    return total;
+}
+
+long oracle_satd_q(const uint8_t *cf, const uint8_t *rf, int W, int H, int x0, int y0, int w, int h, int vx, int vy)
+{
+    return satd_q(cf, rf, W, H, x0, y0, w, h, vx, vy);
+}
+
+int oracle_sme_ex(const uint8_t *cf, const uint8_t *const *rfs, int W, int H, int n_rf, int lambda, int satd,
+                  const int32_t *mb_list, int n_mb, const int16_t *in_mvs,
+                  int16_t *out_qmvs, uint16_t *out_sads, int n_threads);
+
 int oracle_sme_rd(const uint8_t *cf, const uint8_t *const *rfs, int W, int H, int n_rf, int lambda,
+                  const int32_t *mb_list, int n_mb, const int16_t *in_mvs,
+                  int16_t *out_qmvs, uint16_t *out_sads, int n_threads)
+{
+    return oracle_sme_ex(cf, rfs, W, H, n_rf, lambda, 0, mb_list, n_mb, in_mvs, out_qmvs, out_sads, n_threads);
+}
+
+/* metric: SAD (satd = 0, G13) or SATD (satd = 1, G20); outputs the metric value
+ * (not the cost J) of the chosen vector */
+int oracle_sme_ex(const uint8_t *cf, const uint8_t *const *rfs, int W, int H, int n_rf, int lambda, int satd,
                   const int32_t *mb_list, int n_mb, const int16_t *in_mvs,
                   int16_t *out_qmvs, uint16_t *out_sads, int n_threads)
 {
@@ -362,24 +415,27 @@ int oracle_sme_rd(const uint8_t *cf, const uint8_t *const *rfs, int W, int H, in
                 size_t o = ((size_t)i * n_rf + r) * 41 + p;
                 int cx = 4 * in_mvs[2 * o], cy = 4 * in_mvs[2 * o + 1];
                 /* cost J = SADq + lambda * R(v) (G18; lambda = 0: pure SAD, G13) */
-                long bsad = sad_q(cf, rfs[r], W, H, x0, y0, w, h, cx, cy);
+#define DIST(vx, vy) (satd ? satd_q(cf, rfs[r], W, H, x0, y0, w, h, vx, vy) \
+                           : sad_q(cf, rfs[r], W, H, x0, y0, w, h, vx, vy))
+                long bsad = DIST(cx, cy);
                 long best = bsad + (long)lambda * (se_bits(cx) + se_bits(cy));
                 int bx = cx, by = cy;
                 for (int k = 0; k < 8; ++k) {                     /* half-pel ring */
                     int vx = cx + 2 * ring1[k][0], vy = cy + 2 * ring1[k][1];
-                    long s = sad_q(cf, rfs[r], W, H, x0, y0, w, h, vx, vy);
+                    long s = DIST(vx, vy);
                     long j = s + (long)lambda * (se_bits(vx) + se_bits(vy));
                     if (j < best) { best = j; bsad = s; bx = vx; by = vy; }
                 }
                 int qx = bx, qy = by;
                 for (int k = 0; k < 8; ++k) {                     /* quarter-pel ring */
                     int vx = qx + ring1[k][0], vy = qy + ring1[k][1];
-                    long s = sad_q(cf, rfs[r], W, H, x0, y0, w, h, vx, vy);
+                    long s = DIST(vx, vy);
                     long j = s + (long)lambda * (se_bits(vx) + se_bits(vy));
                     if (j < best) { best = j; bsad = s; bx = vx; by = vy; }
                 }
+#undef DIST
                 out_qmvs[2 * o] = (int16_t)bx; out_qmvs[2 * o + 1] = (int16_t)by;
-                out_sads[o] = (uint16_t)bsad;
+                out_sads[o] = (uint16_t)(bsad > 65535 ? 65535 : bsad);   /* SATD can exceed 16 bits (G20) */
             }
     }
     (void)n_threads;

@@ -61,6 +61,7 @@ struct me_ctx {
   int pipeline;          // per-RF ME launches, SME of RF k co-running with ME of RF k+1 (ME_OPT_PIPELINE_RF)
   int me_ctas_per_sm;    // cap on resident ME CTAs per SM (0 = hardware maximum; ME_OPT_ME_CTAS_PER_SM)
   int lambda;            // G18 rate term (ME_OPT_LAMBDA); key = J * kmul + rank
+  int satd;              // G20 SME distortion = Hadamard SATD (ME_OPT_SME_SATD)
   uint32_t kmul;
   int kshift;
   cudaStream_t sme_st;   // pipeline: SME stream
@@ -358,8 +359,14 @@ static int launch_sme(me_ctx* c, const uint8_t* cf, const uint8_t* const* sfs, c
   P.plane = (size_t)c->sf_rows * c->sf_pitch;
   const int warps = n_ref * P.n_rows * P.groups;
   tmark(c, 4, st);
-  if (c->lambda) sme_refine_kernel<true><<<dim3((warps + 3) / 4, 7), 128, 0, st>>>(P);   // y = partition mode
-  else sme_refine_kernel<false><<<dim3((warps + 3) / 4, 7), 128, 0, st>>>(P);
+  const dim3 sg((warps + 3) / 4, 7);   // y = partition mode
+  if (c->satd) {
+    if (c->lambda) sme_refine_kernel<true, true><<<sg, 128, 0, st>>>(P);
+    else sme_refine_kernel<false, true><<<sg, 128, 0, st>>>(P);
+  } else {
+    if (c->lambda) sme_refine_kernel<true, false><<<sg, 128, 0, st>>>(P);
+    else sme_refine_kernel<false, false><<<sg, 128, 0, st>>>(P);
+  }
   tmark(c, 5, st);
   c->last_launches++;
   return launch_status();
@@ -452,7 +459,7 @@ extern "C" int me_encode_frame(me_ctx* c, const uint8_t* cf, const uint8_t* cons
   int st;
   for (int k = 0; k < n_int; ++k)
     if ((st = launch_int(c, rfs[k], sfs[k], c->stream)) != ME_OK) return st;
-  if (c->fuse && !c->lambda)   // ME with the SME fused into the same CTAs (one launch; pure SAD only)
+  if (c->fuse && !c->lambda && !c->satd)   // ME with the SME fused into the same CTAs (one launch; pure SAD only)
     return launch_me(c, cf, rfs, out_mvs, out_sads, c->n_rf, c->stream, reinterpret_cast<const uint8_t* const*>(sfs),
                      out_qmvs, out_qsads);
   return run_me_sme(c, cf, rfs, reinterpret_cast<const uint8_t* const*>(sfs), mvs, sads, out_qmvs, out_qsads, c->n_rf,
@@ -558,7 +565,7 @@ extern "C" int me_stream_push(me_ctx* c, const uint8_t* cf, int cf_on_host, int1
     uint16_t* qs = (out_qsads && !out_on_host) ? out_qsads : (out_on_host ? c->d_qsads2[par] : c->d_qsads);
     // the device output buffer t & 1 is free once the download of push t-2 finished
     if (out_on_host && cudaStreamWaitEvent(c->stream, c->ev_down[par], 0) != cudaSuccess) return launch_status();
-    if (c->fuse && !c->lambda) {
+    if (c->fuse && !c->lambda && !c->satd) {
       // fused: the SME of ref 0 reads SF(t-1), so INT(t-1) runs first on the same stream
       if ((st = launch_int(c, new_rf, new_sf, c->stream)) != ME_OK) return st;
       if ((st = launch_me(c, cur, rfs, nullptr, nullptr, n_ref, c->stream, sfs, qm, qs)) != ME_OK) return st;
@@ -635,6 +642,9 @@ extern "C" int me_set_option(me_ctx* c, int option, int value) {
     case ME_OPT_ME_CTAS_PER_SM:
       if (value < 0 || value > 32) return ME_EINVAL;
       c->me_ctas_per_sm = value;
+      return ME_OK;
+    case ME_OPT_SME_SATD:
+      c->satd = value ? 1 : 0;
       return ME_OK;
     case ME_OPT_LAMBDA:
       if (value < 0 || value > 2000) return ME_EINVAL;

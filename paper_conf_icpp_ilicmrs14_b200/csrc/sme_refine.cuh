@@ -56,6 +56,50 @@ __device__ __forceinline__ uint32_t strip_block_sad(const uint8_t* __restrict__ 
   return s;
 }
 
+// G20: SATD of one 4x4 block = (sum |H D H^T| + 1) >> 1, D = CF - prediction,
+// rows given as packed byte words.  Butterflies (the abs-sum does not depend on
+// the Hadamard row order).
+__device__ __forceinline__ uint32_t satd4(const uint32_t* cfr, const uint32_t* smp) {
+  int t[4][4];
+#pragma unroll
+  for (int r = 0; r < 4; ++r) {
+    int d[4];
+#pragma unroll
+    for (int i = 0; i < 4; ++i) d[i] = (int)((cfr[r] >> (8 * i)) & 0xffu) - (int)((smp[r] >> (8 * i)) & 0xffu);
+    const int s01 = d[0] + d[1], d01 = d[0] - d[1], s23 = d[2] + d[3], d23 = d[2] - d[3];
+    t[r][0] = s01 + s23; t[r][1] = s01 - s23; t[r][2] = d01 - d23; t[r][3] = d01 + d23;
+  }
+  int sum = 0;
+#pragma unroll
+  for (int c = 0; c < 4; ++c) {
+    const int s01 = t[0][c] + t[1][c], d01 = t[0][c] - t[1][c], s23 = t[2][c] + t[3][c], d23 = t[2][c] - t[3][c];
+    sum += abs(s01 + s23) + abs(s01 - s23) + abs(d01 - d23) + abs(d01 + d23);
+  }
+  return (uint32_t)((sum + 1) >> 1);
+}
+
+// SATD of this lane's 4x4 block vs SF samples at quarter offset v (loads as strip_block_sad)
+__device__ __forceinline__ uint32_t strip_block_satd(const uint8_t* __restrict__ sf, size_t plane, int pitch, int pad,
+                                                     int xs, int ys, int vx, int vy, const uint32_t* cfr) {
+  const uint8_t* pl = sf + (size_t)(4 * (vy & 3) + (vx & 3)) * plane;
+  const uint8_t* p0 = pl + (size_t)(ys + (vy >> 2) + pad) * pitch + (xs + (vx >> 2) + pad);
+  const uintptr_t a = reinterpret_cast<uintptr_t>(p0);
+  const uint32_t* w = reinterpret_cast<const uint32_t*>(a & ~uintptr_t(3));
+  const uint32_t sh = 8u * (uint32_t)(a & 3);
+  const int wp = pitch >> 2;
+  uint32_t smp[4];
+#pragma unroll
+  for (int r = 0; r < 4; ++r) smp[r] = __funnelshift_r(__ldg(w + r * wp), __ldg(w + r * wp + 1), sh);
+  return satd4(cfr, smp);
+}
+
+template <bool SATD>
+__device__ __forceinline__ uint32_t strip_block_dist(const uint8_t* __restrict__ sf, size_t plane, int pitch, int pad,
+                                                     int xs, int ys, int vx, int vy, const uint32_t* cfr) {
+  return SATD ? strip_block_satd(sf, plane, pitch, pad, xs, ys, vx, vy, cfr)
+              : strip_block_sad(sf, plane, pitch, pad, xs, ys, vx, vy, cfr);
+}
+
 template <int XMASK>
 __device__ __forceinline__ uint32_t xsum(uint32_t v) {   // all-reduce over the bx lane bits in XMASK
   if (XMASK & 1) v += __shfl_xor_sync(0xffffffffu, v, 1);
@@ -92,8 +136,8 @@ __device__ __forceinline__ int mode_part(int bx, int by) {
 // Axis neighbour (dx,0) = avg(HP(0,0), HP(dx,0)), (0,dy) likewise; diagonal
 // (dx,dy) = avg of the two corners of the half-grid unit square that have one
 // odd coordinate: (0,0) & (dx,dy) if H has mixed parity, else (dx,0) & (0,dy).
-// RD = rate term (G18) compiled in
-template <int MODE, int YG, int XMASK, bool RD>
+// RD = rate term (G18) compiled in; SATD = Hadamard distortion (G20) instead of SAD
+template <int MODE, int YG, int XMASK, bool RD, bool SATD>
 __device__ __forceinline__ void refine_mode(const SmeParams& P, const uint8_t* __restrict__ sf, size_t o, int bx,
                                             int xs, int ys0, bool writer, const uint32_t (&cfs)[16]) {
   constexpr int NG = 4 / YG;           // partitions (block groups) inside this lane's strip
@@ -105,14 +149,14 @@ __device__ __forceinline__ void refine_mode(const SmeParams& P, const uint8_t* _
     const uint32_t mv = __ldg(P.in_mvs + o + p);
     bvx[g] = 4 * (int)(int16_t)(mv & 0xffffu);
     bvy[g] = 4 * (int)(int16_t)(mv >> 16);
-    if (P.in_sads) {
+    if (P.in_sads && !SATD) {
       best[g] = __ldg(P.in_sads + o + p);
     } else {
       uint32_t s = 0;
 #pragma unroll
       for (int j = 0; j < YG; ++j)
-        s += strip_block_sad(sf, P.plane, P.pitch, P.pad, xs, ys0 + 4 * (g * YG + j), bvx[g], bvy[g],
-                             cfs + 4 * (g * YG + j));
+        s += strip_block_dist<SATD>(sf, P.plane, P.pitch, P.pad, xs, ys0 + 4 * (g * YG + j), bvx[g], bvy[g],
+                                    cfs + 4 * (g * YG + j));
       best[g] = xsum<XMASK>(s);
     }
     if (RD) best[g] += P.lambda * (se_bits(bvx[g]) + se_bits(bvy[g]));   // J at the centre
@@ -130,8 +174,8 @@ __device__ __forceinline__ void refine_mode(const SmeParams& P, const uint8_t* _
         uint32_t t = 0;
 #pragma unroll
         for (int j = 0; j < YG; ++j)
-          t += strip_block_sad(sf, P.plane, P.pitch, P.pad, xs, ys0 + 4 * (g * YG + j), ox[g] + 2 * c_ring1[k][0],
-                               oy[g] + 2 * c_ring1[k][1], cfs + 4 * (g * YG + j));
+          t += strip_block_dist<SATD>(sf, P.plane, P.pitch, P.pad, xs, ys0 + 4 * (g * YG + j),
+                                      ox[g] + 2 * c_ring1[k][0], oy[g] + 2 * c_ring1[k][1], cfs + 4 * (g * YG + j));
         sad[k][g] = t;
       }
 #pragma unroll
@@ -160,28 +204,58 @@ __device__ __forceinline__ void refine_mode(const SmeParams& P, const uint8_t* _
 #pragma unroll
     for (int k = 0; k < 8; ++k) qs[k] = 0;
     const uint8_t* rowp = sf + (size_t)(ys0 + 4 * g * YG + P.pad) * P.pitch + (xs + P.pad);
+    if (!SATD) {                                           // SAD: accumulate row by row
 #pragma unroll 1
-    for (int rr = 0; rr < 4 * YG; ++rr, rowp += P.pitch) {
-      uint32_t hp[3][3];
+      for (int rr = 0; rr < 4 * YG; ++rr, rowp += P.pitch) {
+        uint32_t hp[3][3];
 #pragma unroll
-      for (int b = 0; b < 3; ++b)
+        for (int b = 0; b < 3; ++b)
 #pragma unroll
-        for (int a = 0; a < 3; ++a) {
-          const uintptr_t ad = reinterpret_cast<uintptr_t>(rowp + off[b][a]);
-          const uint32_t* w = reinterpret_cast<const uint32_t*>(ad & ~uintptr_t(3));
-          hp[b][a] = __funnelshift_r(__ldg(w), __ldg(w + 1), 8u * (uint32_t)(ad & 3));
+          for (int a = 0; a < 3; ++a) {
+            const uintptr_t ad = reinterpret_cast<uintptr_t>(rowp + off[b][a]);
+            const uint32_t* w = reinterpret_cast<const uint32_t*>(ad & ~uintptr_t(3));
+            hp[b][a] = __funnelshift_r(__ldg(w), __ldg(w + 1), 8u * (uint32_t)(ad & 3));
+          }
+        const uint32_t c = load4_clamped(P.cf, P.W, P.H, xs, ys0 + 4 * g * YG + rr);   // L1 hit
+#pragma unroll
+        for (int k = 0; k < 8; ++k) {
+          const int dx = c_ring1[k][0], dy = c_ring1[k][1];
+          uint32_t v;
+          if (dx == 0 || dy == 0) {
+            v = vavg4(hp[1][1], hp[1 + dy][1 + dx]);
+          } else {
+            v = vavg4(mixed ? hp[1][1] : hp[1][1 + dx], mixed ? hp[1 + dy][1 + dx] : hp[1 + dy][1]);
+          }
+          qs[k] = vad4(c, v, qs[k]);
         }
-      const uint32_t c = load4_clamped(P.cf, P.W, P.H, xs, ys0 + 4 * g * YG + rr);   // L1 hit
+      }
+    } else {                                               // SATD: whole 4x4 blocks, one candidate at a time
+#pragma unroll 1
+      for (int jb = 0; jb < YG; ++jb, rowp += 4 * P.pitch) {
+        uint32_t cw[4];
 #pragma unroll
-      for (int k = 0; k < 8; ++k) {
-        const int dx = c_ring1[k][0], dy = c_ring1[k][1];
-        uint32_t smp;
-        if (dx == 0 || dy == 0) {
-          smp = vavg4(hp[1][1], hp[1 + dy][1 + dx]);
-        } else {
-          smp = vavg4(mixed ? hp[1][1] : hp[1][1 + dx], mixed ? hp[1 + dy][1 + dx] : hp[1 + dy][1]);
+        for (int r = 0; r < 4; ++r) cw[r] = load4_clamped(P.cf, P.W, P.H, xs, ys0 + 4 * (g * YG + jb) + r);
+#pragma unroll 1
+        for (int k = 0; k < 8; ++k) {
+          const int dx = c_ring1[k][0], dy = c_ring1[k][1];
+          // the two half-grid windows this quarter candidate averages (O2 rule, see above)
+          int b0, a0, b1, a1;
+          if (dx == 0 || dy == 0) { b0 = 1; a0 = 1; b1 = 1 + dy; a1 = 1 + dx; }
+          else if (mixed) { b0 = 1; a0 = 1; b1 = 1 + dy; a1 = 1 + dx; }
+          else { b0 = 1; a0 = 1 + dx; b1 = 1 + dy; a1 = 1; }
+          uint32_t smp[4];
+#pragma unroll
+          for (int r = 0; r < 4; ++r) {
+            const uint8_t* rp = rowp + r * P.pitch;
+            const uintptr_t e0 = reinterpret_cast<uintptr_t>(rp + off[b0][a0]);
+            const uintptr_t e1 = reinterpret_cast<uintptr_t>(rp + off[b1][a1]);
+            const uint32_t* w0 = reinterpret_cast<const uint32_t*>(e0 & ~uintptr_t(3));
+            const uint32_t* w1 = reinterpret_cast<const uint32_t*>(e1 & ~uintptr_t(3));
+            smp[r] = vavg4(__funnelshift_r(__ldg(w0), __ldg(w0 + 1), 8u * (uint32_t)(e0 & 3)),
+                           __funnelshift_r(__ldg(w1), __ldg(w1 + 1), 8u * (uint32_t)(e1 & 3)));
+          }
+          qs[k] += satd4(cw, smp);
         }
-        qs[k] = vad4(c, smp, qs[k]);
       }
     }
     const int ox = bvx[g], oy = bvy[g];
@@ -198,12 +272,13 @@ __device__ __forceinline__ void refine_mode(const SmeParams& P, const uint8_t* _
     for (int g = 0; g < NG; ++g) {
       const int p = mode_part<MODE>(bx, g * YG);
       P.out_qmvs[o + p] = (uint32_t)(uint16_t)bvx[g] | ((uint32_t)(uint16_t)bvy[g] << 16);
-      P.out_sads[o + p] = (uint16_t)(best[g] - (RD ? P.lambda * (se_bits(bvx[g]) + se_bits(bvy[g])) : 0));
+      const uint32_t d = best[g] - (RD ? P.lambda * (se_bits(bvx[g]) + se_bits(bvy[g])) : 0);
+      P.out_sads[o + p] = (uint16_t)min(d, 65535u);        // SATD can exceed 16 bits (G20)
     }
   }
 }
 
-template <bool RD>
+template <bool RD, bool SATD>
 __global__ void __launch_bounds__(128) sme_refine_kernel(const SmeParams P) {
   const int warp_id = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
   const int n_warps = P.n_rf * P.n_rows * P.groups;
@@ -224,13 +299,13 @@ __global__ void __launch_bounds__(128) sme_refine_kernel(const SmeParams P) {
   const uint8_t* __restrict__ sf = P.sf[ref];
   const size_t o = ((size_t)(mrow * P.mb_cols + mbx) * P.rf_stride + ref) * kNPart;
   switch (blockIdx.y) {   // one mode per warp: 7x the independent warps (the kernel is latency-bound)
-    case 0: refine_mode<0, 4, 3, RD>(P, sf, o, bx, xs, ys0, writer, cfs); break;   // 16x16
-    case 1: refine_mode<1, 2, 3, RD>(P, sf, o, bx, xs, ys0, writer, cfs); break;   // 16x8
-    case 2: refine_mode<2, 4, 1, RD>(P, sf, o, bx, xs, ys0, writer, cfs); break;   // 8x16
-    case 3: refine_mode<3, 2, 1, RD>(P, sf, o, bx, xs, ys0, writer, cfs); break;   // 8x8
-    case 4: refine_mode<4, 1, 1, RD>(P, sf, o, bx, xs, ys0, writer, cfs); break;   // 8x4
-    case 5: refine_mode<5, 2, 0, RD>(P, sf, o, bx, xs, ys0, writer, cfs); break;   // 4x8
-    default: refine_mode<6, 1, 0, RD>(P, sf, o, bx, xs, ys0, writer, cfs); break;  // 4x4
+    case 0: refine_mode<0, 4, 3, RD, SATD>(P, sf, o, bx, xs, ys0, writer, cfs); break;   // 16x16
+    case 1: refine_mode<1, 2, 3, RD, SATD>(P, sf, o, bx, xs, ys0, writer, cfs); break;   // 16x8
+    case 2: refine_mode<2, 4, 1, RD, SATD>(P, sf, o, bx, xs, ys0, writer, cfs); break;   // 8x16
+    case 3: refine_mode<3, 2, 1, RD, SATD>(P, sf, o, bx, xs, ys0, writer, cfs); break;   // 8x8
+    case 4: refine_mode<4, 1, 1, RD, SATD>(P, sf, o, bx, xs, ys0, writer, cfs); break;   // 8x4
+    case 5: refine_mode<5, 2, 0, RD, SATD>(P, sf, o, bx, xs, ys0, writer, cfs); break;   // 4x8
+    default: refine_mode<6, 1, 0, RD, SATD>(P, sf, o, bx, xs, ys0, writer, cfs); break;  // 4x4
   }
 }
 

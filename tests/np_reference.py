@@ -224,3 +224,55 @@ def mode_decision(qmvs, sads, lam):
         out[i, :9] = res
         out[i, 9] = cost
     return out
+
+
+def satd4_blocks(D):
+    """SATD of an [h, w] difference array (h, w multiples of 4): sum over 4x4 blocks of
+    (sum |Hd D Hd^T| + 1) >> 1 with the Sylvester Hadamard matrix from scipy (rows in
+    another order than the oracle's; the abs-sum does not depend on it)"""
+    from scipy.linalg import hadamard
+    Hd = hadamard(4)
+    tot = 0
+    for by in range(0, D.shape[0], 4):
+        for bx in range(0, D.shape[1], 4):
+            T = Hd @ D[by:by + 4, bx:bx + 4] @ Hd.T
+            tot += (int(np.abs(T).sum()) + 1) >> 1
+    return tot
+
+
+def sme_satd(cf, rfs, mvs, S, lam=0):
+    H, W = cf.shape
+    mbc, mbr = -(-W // 16), -(-H // 16)
+    Wp, Hp = 16 * mbc, 16 * mbr
+    pad = S // 2 + 8
+    pitch, rows = Wp + 2 * pad, Hp + 2 * pad
+    cfp = _edge(cf, ((0, Hp - H), (0, Wp - W)))
+    parts = partitions()
+    qmvs = np.zeros_like(mvs)
+    out = np.zeros(mvs.shape[:3], np.uint16)
+    for r, rf in enumerate(rfs):
+        P = planes(rf, pad, pitch, rows).astype(np.int64)
+        for o in range(mbr * mbc):
+            mby, mbx = divmod(o, mbc)
+            for p, (ox, oy, w, h) in enumerate(parts):
+                x0, y0 = 16 * mbx + ox, 16 * mby + oy
+                blk = cfp[y0:y0 + h, x0:x0 + w]
+
+                def cost(vx, vy):
+                    ph = 4 * (vy & 3) + (vx & 3)
+                    yy, xx = y0 + (vy >> 2) + pad, x0 + (vx >> 2) + pad
+                    d = satd4_blocks(blk - P[ph, yy:yy + h, xx:xx + w])
+                    return d + lam * (se_bits(vx) + se_bits(vy)), d
+
+                c = (4 * int(mvs[o, r, p, 0]), 4 * int(mvs[o, r, p, 1]))
+                (best, bd), bv = cost(*c), c
+                for ring_step in (2, 1):
+                    ctr = bv
+                    for sx, sy in RING1:
+                        v = (ctr[0] + ring_step * sx, ctr[1] + ring_step * sy)
+                        j, d = cost(*v)
+                        if j < best:
+                            best, bd, bv = j, d, v
+                qmvs[o, r, p] = bv
+                out[o, r, p] = bd
+    return qmvs, out

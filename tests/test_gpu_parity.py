@@ -351,3 +351,25 @@ def test_rate_term_me_sme_and_mode_decision(feves, orc, lam, S):
     o_m0, o_s0 = orc.me(cf, rfs, S)
     np.testing.assert_array_equal(m0.cpu().numpy().reshape(n, n_rf, 41, 2), o_m0)
     me.close()
+
+
+@pytest.mark.parametrize("lam,S,kind", [(0, 16, "tex"), (6, 32, "noise"), (0, 8, "flat")])
+def test_sme_satd(feves, orc, lam, S, kind):
+    """f4 (G20): Hadamard-SATD SME on the GPU == oracle (with and without the rate term)"""
+    W, H, n_rf = 64, 48, 2
+    cf, rfs = _frames(kind, W, H, n_rf, 77 + S)
+    me = feves.MotionEstimator(W, H, S, n_rf)
+    me.set_sme_satd(True)
+    if lam:
+        me.set_lambda(lam)
+    tcf, trfs = _dev(cf), [_dev(r) for r in rfs]
+    sfs = [me.new_sf() for _ in trfs]
+    (m, s), (q, qs) = me.encode_frame(tcf, trfs, sfs, n_int=n_rf, out_me=me.new_mvs())
+    torch.cuda.synchronize()
+    n = me.mb_rows * me.mb_cols
+    o_m, _ = orc.me(cf, rfs, S, lam=lam)
+    o_q, o_qs = orc.sme(cf, rfs, o_m, lam=lam, satd=True)
+    np.testing.assert_array_equal(m.cpu().numpy().reshape(n, n_rf, 41, 2), o_m)
+    np.testing.assert_array_equal(qs.cpu().numpy().reshape(n, n_rf, 41), o_qs)
+    np.testing.assert_array_equal(q.cpu().numpy().reshape(n, n_rf, 41, 2), o_q)
+    me.close()

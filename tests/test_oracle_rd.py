@@ -102,3 +102,36 @@ def test_p14_lambda0_never_beats_finest(orc):
     for i in range(out.shape[0]):
         finest = sum(int(s[i, :, 25 + 4 * b:29 + 4 * b].astype(np.int64).sum(axis=1).min()) for b in range(4))
         assert out[i, 9] <= finest
+
+
+# ------------------------------------------------------------------ P15: SATD --
+
+def test_p15_satd_closed_forms(orc):
+    # D constant c on a 4x4 block: H D H^T has only the DC term 16c -> (16|c| + 1) >> 1 = 8|c|
+    rf = np.full((16, 16), 100, np.uint8)
+    for c in (0, 1, 7, -5):
+        cf = np.full((16, 16), 100 + c, np.uint8)
+        assert orc.satd_q(cf, rf, 0, 0, 4, 4, 0, 0) == 8 * abs(c)
+        assert orc.satd_q(cf, rf, 0, 0, 16, 16, 0, 0) == 16 * 8 * abs(c)       # 16 blocks
+    # single impulse d in a block: every coefficient is +-d -> (16|d| + 1) >> 1 = 8|d|
+    cf = rf.copy()
+    cf[1, 2] = 100 + 9
+    assert orc.satd_q(cf, rf, 0, 0, 4, 4, 0, 0) == 72
+    # odd total: one coefficient pattern giving sum 2k+1 is impossible for integer D (all
+    # coefficients share parity), so (s+1)>>1 == s/2 here; a 2-pixel difference d,-d in one row
+    cf = rf.copy()
+    cf[0, 0], cf[0, 1] = 103, 97            # D row 0 = (3, -3, 0, 0)
+    assert orc.satd_q(cf, rf, 0, 0, 4, 4, 0, 0) == (sum(abs(v) for v in (0, 0, 6, 6)) * 4 + 1) // 2
+
+
+def test_p15_satd_sme_vs_numpy(orc):
+    cf, rf0 = gen_tex(32, 32, 1, 8), gen_tex(32, 32, 0, 8)
+    mvs, _ = orc.me(cf, [rf0], 8)
+    qo, so = orc.sme(cf, [rf0], mvs, satd=True)
+    qn, sn = npr.sme_satd(cf, [rf0], mvs, 8)
+    np.testing.assert_array_equal(qo, qn)
+    np.testing.assert_array_equal(so, sn)
+    qo2, so2 = orc.sme(cf, [rf0], mvs, satd=True, lam=5)
+    qn2, sn2 = npr.sme_satd(cf, [rf0], mvs, 8, lam=5)
+    np.testing.assert_array_equal(qo2, qn2)
+    np.testing.assert_array_equal(so2, sn2)
