@@ -213,7 +213,11 @@ class MotionEstimator:
         """SME fused into the ME kernel (default) or as its own launch."""
         _check(lib().me_set_fused(self._ctx, int(on)))
 
-    OPT_FUSED_SME, OPT_PIPELINE_RF, OPT_ME_CTAS_PER_SM, OPT_LAMBDA, OPT_SME_SATD = 1, 2, 3, 4, 5
+    OPT_FUSED_SME, OPT_PIPELINE_RF, OPT_ME_CTAS_PER_SM, OPT_LAMBDA, OPT_SME_SATD, OPT_SA_INCLUSIVE = 1, 2, 3, 4, 5, 6
+
+    def set_sa_inclusive(self, on: bool = True):
+        """Candidates in [-S/2, +S/2]^2 (G1 alternative reading, f4)."""
+        self.set_option(self.OPT_SA_INCLUSIVE, int(on))
 
     def set_sme_satd(self, on: bool = True):
         """SME distortion = 4x4 Hadamard SATD (f4, G20) instead of SAD."""

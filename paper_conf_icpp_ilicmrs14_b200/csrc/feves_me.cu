@@ -62,6 +62,7 @@ struct me_ctx {
   int me_ctas_per_sm;    // cap on resident ME CTAs per SM (0 = hardware maximum; ME_OPT_ME_CTAS_PER_SM)
   int lambda;            // G18 rate term (ME_OPT_LAMBDA); key = J * kmul + rank
   int satd;              // G20 SME distortion = Hadamard SATD (ME_OPT_SME_SATD)
+  int inclusive;         // G1 alternative: candidates [-R, R]^2 (ME_OPT_SA_INCLUSIVE)
   uint32_t kmul;
   int kshift;
   cudaStream_t sme_st;   // pipeline: SME stream
@@ -115,15 +116,24 @@ static int launch_status() {
 // term J = SAD + lambda*R may exceed 16 bits, so key = J * 2^15 + rank (rank < 2^15
 // for S <= 128, J < 2^17 for lambda <= 2000).
 static int upload_key_table(me_ctx* c) {
-  const int S = c->S;
+  const int Sc = c->S + c->inclusive, hi = Sc - 1 - c->R;   // candidates per axis, dx,dy in [-R, hi]
   c->kshift = c->lambda ? 15 : 16;
   c->kmul = 1u << c->kshift;
-  std::vector<uint32_t> e((size_t)S * S);
-  for (int dy = -c->R; dy < c->R; ++dy)
-    for (int dx = -c->R; dx < c->R; ++dx)
-      e[(size_t)(dy + c->R) * S + (dx + c->R)] =
-          (uint32_t)(c->lambda * (se_bits(4 * dx) + se_bits(4 * dy))) * c->kmul + (uint32_t)spiral_rank_closed_form(dx, dy);
-  return cudaMemcpy(c->d_rank, e.data(), e.size() * 4, cudaMemcpyHostToDevice) == cudaSuccess ? ME_OK : ME_ECUDA;
+  std::vector<uint32_t> e((size_t)Sc * Sc), inv((size_t)(c->S + 1) * (c->S + 1), 0);
+  for (int dy = -c->R; dy <= hi; ++dy)
+    for (int dx = -c->R; dx <= hi; ++dx) {
+      const int r = spiral_rank_closed_form(dx, dy);
+      e[(size_t)(dy + c->R) * Sc + (dx + c->R)] =
+          (uint32_t)(c->lambda * (se_bits(4 * dx) + se_bits(4 * dy))) * c->kmul + (uint32_t)r;
+      inv[r] = (uint32_t)(uint16_t)dx | ((uint32_t)(uint16_t)dy << 16);
+    }
+  c->me_threads = me_threads(Sc);
+  c->me_smem = (size_t)me_smem_words(Sc) * 4;
+  c->me_smem_fused = (size_t)me_smem_words_fused(Sc, c->n_rf) * 4;
+  return cudaMemcpy(c->d_rank, e.data(), e.size() * 4, cudaMemcpyHostToDevice) == cudaSuccess &&
+                 cudaMemcpy(c->d_inv, inv.data(), inv.size() * 4, cudaMemcpyHostToDevice) == cudaSuccess
+             ? ME_OK
+             : ME_ECUDA;
 }
 
 // ------------------------------------------------------------ lifetime ----
@@ -152,20 +162,15 @@ extern "C" me_ctx* me_create(int width, int height, int sa_range, int n_rf) {
   c->pipeline = 0;
   c->me_ctas_per_sm = 0;
 
-  std::vector<uint32_t> inv((size_t)(S + 1) * (S + 1), 0);
-  for (int dy = -c->R; dy < c->R; ++dy)
-    for (int dx = -c->R; dx < c->R; ++dx)
-      inv[spiral_rank_closed_form(dx, dy)] = (uint32_t)(uint16_t)dx | ((uint32_t)(uint16_t)dy << 16);
   const size_t nmv = (size_t)c->mb_cols * c->mb_rows * n_rf * kNPart;
-  bool ok = cudaMalloc(&c->d_rank, (size_t)S * S * 4) == cudaSuccess &&
-            cudaMalloc(&c->d_inv, inv.size() * 4) == cudaSuccess &&
+  bool ok = cudaMalloc(&c->d_rank, (size_t)(S + 1) * (S + 1) * 4) == cudaSuccess &&
+            cudaMalloc(&c->d_inv, (size_t)(S + 1) * (S + 1) * 4) == cudaSuccess &&
             cudaMalloc(&c->d_mvs, nmv * 4) == cudaSuccess &&
             cudaMalloc(&c->d_sads, nmv * 2) == cudaSuccess &&
             cudaStreamCreateWithFlags(&c->stream, cudaStreamNonBlocking) == cudaSuccess;
   if (ok) {
     c->own_stream = true;
     ok = upload_key_table(c) == ME_OK &&
-         cudaMemcpy(c->d_inv, inv.data(), inv.size() * 4, cudaMemcpyHostToDevice) == cudaSuccess &&
          set_me_smem(200 * 1024) == cudaSuccess;   // max; the launch asks for what it needs
   }
   if (!ok) {
@@ -268,7 +273,7 @@ static int launch_me(me_ctx* c, const uint8_t* cf, const uint8_t* const* rfs, in
   memset(&P, 0, sizeof(P));
   P.cf = cf;
   for (int k = 0; k < n_ref; ++k) P.rf[k] = rfs[k];
-  P.W = c->W; P.H = c->H; P.S = c->S; P.R = c->R; P.n_rf = n_ref; P.rf_stride = c->n_rf;
+  P.W = c->W; P.H = c->H; P.S = c->S + c->inclusive; P.R = c->R; P.n_rf = n_ref; P.rf_stride = c->n_rf;
   P.mb_cols = c->mb_cols; P.row0 = c->row0;
   P.rank_tab = c->d_rank; P.inv_tab = c->d_inv;
   P.kmul = c->kmul; P.kshift = c->kshift; P.lambda = c->lambda;
@@ -295,7 +300,7 @@ static int launch_me(me_ctx* c, const uint8_t* cf, const uint8_t* const* rfs, in
     else if (c->lambda) me_fsbm_kernel<SS, false, 15><<<grid, c->me_threads, smem, st>>>(P); \
     else me_fsbm_kernel<SS, false><<<grid, c->me_threads, smem, st>>>(P);               \
   } while (0)
-  switch (c->S) {   // compile-time window geometry for the paper's SA sizes (Fig. 6a: 32..256)
+  switch (c->inclusive ? 0 : c->S) {   // compile-time window geometry for the paper's SA sizes (Fig. 6a: 32..256)
     case 16: FEVES_ME_LAUNCH(16); break;
     case 32: FEVES_ME_LAUNCH(32); break;
     case 64: FEVES_ME_LAUNCH(64); break;
@@ -459,7 +464,7 @@ extern "C" int me_encode_frame(me_ctx* c, const uint8_t* cf, const uint8_t* cons
   int st;
   for (int k = 0; k < n_int; ++k)
     if ((st = launch_int(c, rfs[k], sfs[k], c->stream)) != ME_OK) return st;
-  if (c->fuse && !c->lambda && !c->satd)   // ME with the SME fused into the same CTAs (one launch; pure SAD only)
+  if (c->fuse && !c->lambda && !c->satd && !c->inclusive)   // ME with the SME fused (one launch; base reading only)
     return launch_me(c, cf, rfs, out_mvs, out_sads, c->n_rf, c->stream, reinterpret_cast<const uint8_t* const*>(sfs),
                      out_qmvs, out_qsads);
   return run_me_sme(c, cf, rfs, reinterpret_cast<const uint8_t* const*>(sfs), mvs, sads, out_qmvs, out_qsads, c->n_rf,
@@ -565,7 +570,7 @@ extern "C" int me_stream_push(me_ctx* c, const uint8_t* cf, int cf_on_host, int1
     uint16_t* qs = (out_qsads && !out_on_host) ? out_qsads : (out_on_host ? c->d_qsads2[par] : c->d_qsads);
     // the device output buffer t & 1 is free once the download of push t-2 finished
     if (out_on_host && cudaStreamWaitEvent(c->stream, c->ev_down[par], 0) != cudaSuccess) return launch_status();
-    if (c->fuse && !c->lambda && !c->satd) {
+    if (c->fuse && !c->lambda && !c->satd && !c->inclusive) {
       // fused: the SME of ref 0 reads SF(t-1), so INT(t-1) runs first on the same stream
       if ((st = launch_int(c, new_rf, new_sf, c->stream)) != ME_OK) return st;
       if ((st = launch_me(c, cur, rfs, nullptr, nullptr, n_ref, c->stream, sfs, qm, qs)) != ME_OK) return st;
@@ -643,6 +648,10 @@ extern "C" int me_set_option(me_ctx* c, int option, int value) {
       if (value < 0 || value > 32) return ME_EINVAL;
       c->me_ctas_per_sm = value;
       return ME_OK;
+    case ME_OPT_SA_INCLUSIVE:
+      if (c->stream) cudaStreamSynchronize(c->stream);   // the tables may be in use
+      c->inclusive = value ? 1 : 0;
+      return upload_key_table(c);
     case ME_OPT_SME_SATD:
       c->satd = value ? 1 : 0;
       return ME_OK;

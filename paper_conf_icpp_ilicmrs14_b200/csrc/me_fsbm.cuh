@@ -34,10 +34,11 @@ constexpr int kMeT = 4;   // candidates per vertical step
 struct MeParams {
   const uint8_t* cf;
   const uint8_t* rf[kMaxRf];
-  int W, H, S, R, n_rf;       // n_rf = RFs searched by this launch (RF ramp)
+  int W, H, S, R, n_rf;       // S = candidates per axis (sa_range, +1 if inclusive); n_rf = RFs searched
   int rf_stride;              // RF dimension of the output layout (the context's n_rf)
   int mb_cols, row0;
-  const uint32_t* rank_tab;   // [S][S], [dy+R][dx+R] -> key addend E = lambda*R(4dx,4dy)*kmul + spiral rank (G4, G18)
+  const uint32_t* rank_tab;   // [S][S] (S candidates per axis), [dy+R][dx+R] -> key addend E =
+                              // lambda*R(4dx,4dy)*kmul + spiral rank (G4, G18)
   const uint32_t* inv_tab;    // rank -> (dx & 0xffff) | (dy << 16)
   uint32_t kmul;              // key = J * kmul + rank: 2^16 (lambda = 0) or 2^15 (J may exceed 16 bits)
   int kshift, lambda;
@@ -275,10 +276,15 @@ __device__ __forceinline__ void fused_sme(const MeParams& P, const uint32_t* cf_
 // FUSE = also run the SME of this MB (fused_sme) after its ME;
 // KSH = key shift: 16 (pure SAD) or 15 (rate term, G18: J may exceed 16 bits).
 template <int S_CT, bool FUSE = false, int KSH = 16>
-__global__ void __launch_bounds__(128, 4) me_fsbm_kernel(const MeParams P) {
+// S_CT > 0: <= 128 candidates/axis -> <= 4 warps, 4 CTAs/SM.  S_CT == 0 (runtime S,
+// incl. the inclusive SA's 129 candidates -> 5 warps): same 128-register cap.
+__global__ void __launch_bounds__(S_CT ? 128 : 256, S_CT ? 4 : 2) me_fsbm_kernel(const MeParams P) {
   extern __shared__ __align__(16) uint32_t smem[];
+  // S = candidates per axis: sa_range (G1), or sa_range + 1 for the inclusive SA (f4);
+  // candidates dx, dy in [-R, hi], hi = S - 1 - R (R - 1, or R when inclusive)
   const int S = S_CT ? S_CT : P.S;
-  const int R = S / 2;
+  const int R = S_CT ? S_CT / 2 : P.R;
+  const int hi = S - 1 - R;
   const int PW = me_pw(S), CSTRIDE = me_cstride(S), LX = me_lx(S), NGX = me_ngx(S);
   const int NSUB = me_nsub(S), DYL = me_dyl(S);
   uint32_t* cf_s = smem;                                  // 16 rows x 4 words
@@ -295,7 +301,7 @@ __global__ void __launch_bounds__(128, 4) me_fsbm_kernel(const MeParams P) {
   // ---- lane geometry: dx column and dy sub-range ----
   const int gx = warp % NGX;
   const int xi = lane % LX, sub = lane / LX;
-  const int dx = min(-R + gx * LX + xi, R - 1);            // beyond-range lanes duplicate dx=R-1
+  const int dx = min(-R + gx * LX + xi, hi);               // beyond-range lanes duplicate dx=hi
   const int off = dx + R;                                  // byte offset inside the window row
   const uint32_t* wbase = win + (off & 3) * CSTRIDE + (off >> 2);
   const int dy_begin = -R + sub * DYL;
@@ -351,17 +357,17 @@ __global__ void __launch_bounds__(128, 4) me_fsbm_kernel(const MeParams P) {
     const uint32_t* rank_col = P.rank_tab + off;
     uint32_t rank_next[kMeT];
     {
-      const int dy0 = min(dy_begin, R - kMeT);
+      const int dy0 = min(dy_begin, hi + 1 - kMeT);
 #pragma unroll
       for (int t = 0; t < kMeT; ++t) rank_next[t] = __ldg(rank_col + (dy0 + t + R) * S);
     }
     for (int c = 0; c < DYL; c += kMeT) {
-      const int dy0 = min(dy_begin + c, R - kMeT);        // clamped chunk: duplicates are harmless
+      const int dy0 = min(dy_begin + c, hi + 1 - kMeT);   // clamped chunk: duplicates are harmless
       uint32_t rank[kMeT];
 #pragma unroll
       for (int t = 0; t < kMeT; ++t) rank[t] = rank_next[t];
       {                                                   // prefetch the next chunk's ranks
-        const int dn = min(dy_begin + c + kMeT, R - kMeT);
+        const int dn = min(dy_begin + c + kMeT, hi + 1 - kMeT);
 #pragma unroll
         for (int t = 0; t < kMeT; ++t) rank_next[t] = __ldg(rank_col + (dn + t + R) * S);
       }

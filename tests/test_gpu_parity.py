@@ -373,3 +373,35 @@ def test_sme_satd(feves, orc, lam, S, kind):
     np.testing.assert_array_equal(qs.cpu().numpy().reshape(n, n_rf, 41), o_qs)
     np.testing.assert_array_equal(q.cpu().numpy().reshape(n, n_rf, 41, 2), o_q)
     me.close()
+
+
+@pytest.mark.parametrize("W,H,S,n_rf,kind,lam", [
+    (64, 48, 16, 2, "tex", 0), (72, 52, 32, 1, "noise", 0), (40, 40, 128, 1, "noise", 0),
+    (50, 30, 6, 1, "flat", 0), (80, 48, 64, 2, "tex", 0), (64, 48, 16, 2, "tex", 9)])
+def test_sa_inclusive(feves, orc, W, H, S, n_rf, kind, lam):
+    """f4 (G1 alternative reading): candidates [-S/2, +S/2]^2 on the GPU == oracle(sa_inclusive=True),
+    then SME on those MVs; switching back restores the base reading's results"""
+    cf, rfs = _frames(kind, W, H, n_rf, 500 + S + lam)
+    me = feves.MotionEstimator(W, H, S, n_rf)
+    me.set_sa_inclusive(True)
+    if lam:
+        me.set_lambda(lam)
+    tcf, trfs = _dev(cf), [_dev(r) for r in rfs]
+    sfs = [me.new_sf() for _ in trfs]
+    (m, s), (q, qs) = me.encode_frame(tcf, trfs, sfs, n_int=n_rf, out_me=me.new_mvs())
+    torch.cuda.synchronize()
+    n = me.mb_rows * me.mb_cols
+    o_m, o_s = orc.me(cf, rfs, S, sa_inclusive=True, lam=lam)
+    np.testing.assert_array_equal(m.cpu().numpy().reshape(n, n_rf, 41, 2), o_m)
+    np.testing.assert_array_equal(s.cpu().numpy().reshape(n, n_rf, 41), o_s)
+    assert np.abs(o_m).max() <= S // 2
+    o_q, o_qs = orc.sme(cf, rfs, o_m, lam=lam)
+    np.testing.assert_array_equal(q.cpu().numpy().reshape(n, n_rf, 41, 2), o_q)
+    np.testing.assert_array_equal(qs.cpu().numpy().reshape(n, n_rf, 41), o_qs)
+    me.set_sa_inclusive(False)
+    (m0, s0), _ = me.encode_frame(tcf, trfs, sfs, n_int=0, out_me=me.new_mvs())
+    torch.cuda.synchronize()
+    o_m0, o_s0 = orc.me(cf, rfs, S, lam=lam)
+    np.testing.assert_array_equal(m0.cpu().numpy().reshape(n, n_rf, 41, 2), o_m0)
+    np.testing.assert_array_equal(s0.cpu().numpy().reshape(n, n_rf, 41), o_s0)
+    me.close()
