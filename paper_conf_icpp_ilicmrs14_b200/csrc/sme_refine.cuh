@@ -100,6 +100,109 @@ __device__ __forceinline__ uint32_t strip_block_dist(const uint8_t* __restrict__
               : strip_block_sad(sf, plane, pitch, pad, xs, ys, vx, vy, cfr);
 }
 
+// Two aligned words holding the 5 bytes at [a, a+5): the 4-byte windows at a
+// (left) and a+1 (right) are both funnel shifts of them (the right one with the
+// clamped shift, 32 -> the high word).  One pair of LDG per row serves the two
+// horizontally adjacent half-grid windows of the SME (same plane, columns x, x+1).
+struct Win2 { uint32_t l, r; };
+__device__ __forceinline__ Win2 load_lr(const uint8_t* __restrict__ p) {
+  const uintptr_t a = reinterpret_cast<uintptr_t>(p);
+  const uint32_t* w = reinterpret_cast<const uint32_t*>(a & ~uintptr_t(3));
+  const uint32_t w0 = __ldg(w), w1 = __ldg(w + 1), sh = 8u * (uint32_t)(a & 3);
+  return {__funnelshift_r(w0, w1, sh), __funnelshift_rc(w0, w1, sh + 8u)};
+}
+__device__ __forceinline__ uint32_t load_w(const uint8_t* __restrict__ p) {
+  const uintptr_t a = reinterpret_cast<uintptr_t>(p);
+  const uint32_t* w = reinterpret_cast<const uint32_t*>(a & ~uintptr_t(3));
+  return __funnelshift_r(__ldg(w), __ldg(w + 1), 8u * (uint32_t)(a & 3));
+}
+
+// Half stage, SAD, one block group of HR rows (DESIGN.md §6 "row sweep"): for the
+// full-pel centre (mx, my) the 8 ring candidates c + 2 s_k are windows of three
+// half-sample planes at integer offsets (phase 4*yFrac + xFrac, G11):
+//   (0,-1) h @ (mx, my-1)    (0,+1) h @ (mx, my)
+//   (-1,-1) j @ (mx-1, my-1) (+1,-1) j @ (mx, my-1)
+//   (-1,0) b @ (mx-1, my)    (+1,0) b @ (mx, my)
+//   (-1,+1) j @ (mx-1, my)   (+1,+1) j @ (mx, my)
+// so sweeping plane rows my-1 .. my+HR-1 once, each h / j row serves a candidate
+// above (CF row r) and one below (CF row r-1), and each j / b row pair of words
+// serves the left and right candidate: 6 LDG per row instead of 16.
+template <int HR>
+__device__ __forceinline__ void half_sad_sweep(const uint8_t* __restrict__ sf, size_t plane, int pitch,
+                                               const uint8_t* base, int mx, int my, const uint32_t* cf,
+                                               uint32_t (&sad)[8]) {
+  // base = plane 0 at the strip's top-left integer sample (pad applied)
+  const uint8_t* ph = base + 8 * plane + (ptrdiff_t)(my - 1) * pitch + mx;
+  const uint8_t* pj = base + 10 * plane + (ptrdiff_t)(my - 1) * pitch + (mx - 1);
+  const uint8_t* pb = base + 2 * plane + (ptrdiff_t)my * pitch + (mx - 1);
+#pragma unroll
+  for (int k = 0; k < 8; ++k) sad[k] = 0;
+#pragma unroll
+  for (int r = 0; r <= HR; ++r) {
+    const uint32_t hw = load_w(ph + r * pitch);
+    const Win2 jw = load_lr(pj + r * pitch);
+    if (r < HR) {
+      const Win2 bw = load_lr(pb + r * pitch);
+      sad[0] = vad4(cf[r], hw, sad[0]);
+      sad[2] = vad4(cf[r], jw.l, sad[2]);
+      sad[3] = vad4(cf[r], jw.r, sad[3]);
+      sad[4] = vad4(cf[r], bw.l, sad[4]);
+      sad[5] = vad4(cf[r], bw.r, sad[5]);
+    }
+    if (r > 0) {
+      sad[1] = vad4(cf[r - 1], hw, sad[1]);
+      sad[6] = vad4(cf[r - 1], jw.l, sad[6]);
+      sad[7] = vad4(cf[r - 1], jw.r, sad[7]);
+    }
+  }
+}
+
+// the 8 quarter candidates around half-grid point H from its 3x3 half-grid
+// windows hp[b][a] (rows hy-1..hy+1, columns hx-1..hx+1), O2 averaging rule
+__device__ __forceinline__ uint32_t quarter_win(const uint32_t (&hp)[3][3], int k, bool mixed) {
+  const int dx = k < 2 ? 0 : ((k & 1) ? 1 : -1);
+  const int dy = k < 2 ? ((k & 1) ? 1 : -1) : (k < 4 ? -1 : k < 6 ? 0 : 1);
+  if (dx == 0 || dy == 0) return vavg4(hp[1][1], hp[1 + dy][1 + dx]);
+  return vavg4(mixed ? hp[1][1] : hp[1][1 + dx], mixed ? hp[1 + dy][1 + dx] : hp[1 + dy][1]);
+}
+
+// Quarter stage, SAD, one block group of HR rows, around half-grid point (hx, hy):
+// half-grid columns hx-1 and hx+1 share a plane and are adjacent integer columns
+// (one load_lr), likewise rows hy-1 and hy+1 are adjacent rows of one plane, so
+// the sweep reads "outer" rows (hy+-1 parity) r = 0..HR and "middle" rows (hy
+// parity) r = 0..HR-1, 4 LDG each, and CF row r uses outer r, middle r, outer r+1.
+template <int HR>
+__device__ __forceinline__ void quarter_sad_sweep(size_t plane, int pitch, const uint8_t* base, int hx, int hy,
+                                                  const uint32_t* cf, uint32_t (&qs)[8]) {
+  const bool mixed = ((hx ^ hy) & 1) != 0;
+  const int xm = hx - 1, x0 = hx, ym = hy - 1, y0 = hy;
+  auto at = [&](int X, int Y) {                 // plane row pointer of half-grid point (X, Y), CF row 0
+    return base + (size_t)(8 * (Y & 1) + 2 * (X & 1)) * plane + (ptrdiff_t)(Y >> 1) * pitch + (X >> 1);
+  };
+  const uint8_t* o_lr = at(xm, ym);             // outer rows, columns hx-1 / hx+1
+  const uint8_t* o_c = at(x0, ym);              // outer rows, column hx
+  const uint8_t* m_lr = at(xm, y0);             // middle rows
+  const uint8_t* m_c = at(x0, y0);
+#pragma unroll
+  for (int k = 0; k < 8; ++k) qs[k] = 0;
+  uint32_t po[3], pm[3];                        // previous outer / middle windows (L, C, R)
+#pragma unroll
+  for (int r = 0; r <= HR; ++r) {
+    const Win2 olr = load_lr(o_lr + r * pitch);
+    const uint32_t oc = load_w(o_c + r * pitch);
+    if (r > 0) {
+      const uint32_t hp[3][3] = {{po[0], po[1], po[2]}, {pm[0], pm[1], pm[2]}, {olr.l, oc, olr.r}};
+#pragma unroll
+      for (int k = 0; k < 8; ++k) qs[k] = vad4(cf[r - 1], quarter_win(hp, k, mixed), qs[k]);
+    }
+    if (r < HR) {
+      const Win2 mlr = load_lr(m_lr + r * pitch);
+      pm[0] = mlr.l; pm[1] = load_w(m_c + r * pitch); pm[2] = mlr.r;
+      po[0] = olr.l; po[1] = oc; po[2] = olr.r;
+    }
+  }
+}
+
 template <int XMASK>
 __device__ __forceinline__ uint32_t xsum(uint32_t v) {   // all-reduce over the bx lane bits in XMASK
   if (XMASK & 1) v += __shfl_xor_sync(0xffffffffu, v, 1);
@@ -161,23 +264,35 @@ __device__ __forceinline__ void refine_mode(const SmeParams& P, const uint8_t* _
     }
     if (RD) best[g] += P.lambda * (se_bits(bvx[g]) + se_bits(bvy[g]));   // J at the centre
   }
-  // ---- half stage (all 8 candidates' loads first: latency-bound) ----
+  // ---- half stage ----
   {
     int ox[NG], oy[NG];
 #pragma unroll
     for (int g = 0; g < NG; ++g) { ox[g] = bvx[g]; oy[g] = bvy[g]; }
     uint32_t sad[8][NG];
-#pragma unroll
-    for (int k = 0; k < 8; ++k)
+    if (!SATD) {                                    // SAD: one row sweep per block group
+      const uint8_t* base = sf + (size_t)(ys0 + P.pad) * P.pitch + (xs + P.pad);
 #pragma unroll
       for (int g = 0; g < NG; ++g) {
-        uint32_t t = 0;
+        uint32_t sg[8];
+        half_sad_sweep<4 * YG>(sf, P.plane, P.pitch, base + (size_t)(4 * g * YG) * P.pitch, ox[g] >> 2, oy[g] >> 2,
+                               cfs + 4 * g * YG, sg);
 #pragma unroll
-        for (int j = 0; j < YG; ++j)
-          t += strip_block_dist<SATD>(sf, P.plane, P.pitch, P.pad, xs, ys0 + 4 * (g * YG + j),
-                                      ox[g] + 2 * c_ring1[k][0], oy[g] + 2 * c_ring1[k][1], cfs + 4 * (g * YG + j));
-        sad[k][g] = t;
+        for (int k = 0; k < 8; ++k) sad[k][g] = sg[k];
       }
+    } else {                                        // SATD: whole 4x4 blocks per candidate
+#pragma unroll
+      for (int k = 0; k < 8; ++k)
+#pragma unroll
+        for (int g = 0; g < NG; ++g) {
+          uint32_t t = 0;
+#pragma unroll
+          for (int j = 0; j < YG; ++j)
+            t += strip_block_dist<SATD>(sf, P.plane, P.pitch, P.pad, xs, ys0 + 4 * (g * YG + j),
+                                        ox[g] + 2 * c_ring1[k][0], oy[g] + 2 * c_ring1[k][1], cfs + 4 * (g * YG + j));
+          sad[k][g] = t;
+        }
+    }
 #pragma unroll
     for (int k = 0; k < 8; ++k)
 #pragma unroll
@@ -204,31 +319,9 @@ __device__ __forceinline__ void refine_mode(const SmeParams& P, const uint8_t* _
 #pragma unroll
     for (int k = 0; k < 8; ++k) qs[k] = 0;
     const uint8_t* rowp = sf + (size_t)(ys0 + 4 * g * YG + P.pad) * P.pitch + (xs + P.pad);
-    if (!SATD) {                                           // SAD: accumulate row by row
-#pragma unroll 1
-      for (int rr = 0; rr < 4 * YG; ++rr, rowp += P.pitch) {
-        uint32_t hp[3][3];
-#pragma unroll
-        for (int b = 0; b < 3; ++b)
-#pragma unroll
-          for (int a = 0; a < 3; ++a) {
-            const uintptr_t ad = reinterpret_cast<uintptr_t>(rowp + off[b][a]);
-            const uint32_t* w = reinterpret_cast<const uint32_t*>(ad & ~uintptr_t(3));
-            hp[b][a] = __funnelshift_r(__ldg(w), __ldg(w + 1), 8u * (uint32_t)(ad & 3));
-          }
-        const uint32_t c = load4_clamped(P.cf, P.W, P.H, xs, ys0 + 4 * g * YG + rr);   // L1 hit
-#pragma unroll
-        for (int k = 0; k < 8; ++k) {
-          const int dx = c_ring1[k][0], dy = c_ring1[k][1];
-          uint32_t v;
-          if (dx == 0 || dy == 0) {
-            v = vavg4(hp[1][1], hp[1 + dy][1 + dx]);
-          } else {
-            v = vavg4(mixed ? hp[1][1] : hp[1][1 + dx], mixed ? hp[1 + dy][1 + dx] : hp[1 + dy][1]);
-          }
-          qs[k] = vad4(c, v, qs[k]);
-        }
-      }
+    if (!SATD) {                                           // SAD: one row sweep
+      quarter_sad_sweep<4 * YG>(P.plane, P.pitch, sf + (size_t)(ys0 + 4 * g * YG + P.pad) * P.pitch + (xs + P.pad),
+                                hx, hy, cfs + 4 * g * YG, qs);
     } else {                                               // SATD: whole 4x4 blocks, one candidate at a time
 #pragma unroll 1
       for (int jb = 0; jb < YG; ++jb, rowp += 4 * P.pitch) {
