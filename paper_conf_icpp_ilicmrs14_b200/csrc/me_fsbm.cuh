@@ -29,7 +29,13 @@
 
 namespace feves {
 
-constexpr int kMeT = 4;   // candidates per vertical step
+#ifndef FEVES_ME_T
+#define FEVES_ME_T 4
+#endif
+#ifndef FEVES_ME_MINB
+#define FEVES_ME_MINB 4
+#endif
+constexpr int kMeT = FEVES_ME_T;   // candidates per vertical step
 
 struct MeParams {
   const uint8_t* cf;
@@ -278,7 +284,7 @@ __device__ __forceinline__ void fused_sme(const MeParams& P, const uint32_t* cf_
 template <int S_CT, bool FUSE = false, int KSH = 16>
 // S_CT > 0: <= 128 candidates/axis -> <= 4 warps, 4 CTAs/SM.  S_CT == 0 (runtime S,
 // incl. the inclusive SA's 129 candidates -> 5 warps): same 128-register cap.
-__global__ void __launch_bounds__(S_CT ? 128 : 256, S_CT ? 4 : 2) me_fsbm_kernel(const MeParams P) {
+__global__ void __launch_bounds__(S_CT ? 128 : 256, S_CT ? FEVES_ME_MINB : 2) me_fsbm_kernel(const MeParams P) {
   extern __shared__ __align__(16) uint32_t smem[];
   // S = candidates per axis: sa_range (G1), or sa_range + 1 for the inclusive SA (f4);
   // candidates dx, dy in [-R, hi], hi = S - 1 - R (R - 1, or R when inclusive)

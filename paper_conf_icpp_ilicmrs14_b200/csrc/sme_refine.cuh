@@ -9,7 +9,9 @@
 //
 // Mapping (L1-sector bound kernel): one warp = 8 horizontally
 // adjacent MBs of one RF x 4 lanes; lane (g, bx) owns the 4-pixel column
-// strip bx of MB g (its four 4x4 blocks by = 0..3, CF strip in 16 registers).
+// strip bx of MB g (its four 4x4 blocks by = 0..3); the lane refines the
+// partitions of its strip one after the other, loading only that partition's
+// CF rows (80 registers -> 24 resident warps per SM for a latency-bound kernel).
 // For one candidate, every LDG of the warp reads one row of 8 x 16 contiguous
 // bytes of one SF phase plane when the MBs' MVs agree (the common case), so a
 // request touches ~5 sectors instead of 16.  A partition's SAD = sum over its
@@ -242,137 +244,122 @@ __device__ __forceinline__ int mode_part(int bx, int by) {
 // RD = rate term (G18) compiled in; SATD = Hadamard distortion (G20) instead of SAD
 template <int MODE, int YG, int XMASK, bool RD, bool SATD>
 __device__ __forceinline__ void refine_mode(const SmeParams& P, const uint8_t* __restrict__ sf, size_t o, int bx,
-                                            int xs, int ys0, bool writer, const uint32_t (&cfs)[16]) {
+                                            int xs, int ys0, bool writer) {
   constexpr int NG = 4 / YG;           // partitions (block groups) inside this lane's strip
-  int bvx[NG], bvy[NG];
-  uint32_t best[NG];
-#pragma unroll
+  // The groups are refined one after the other (latency-bound kernel: fewer live
+  // registers -> more resident warps beats the ILP of refining all NG at once).
+#pragma unroll 1
   for (int g = 0; g < NG; ++g) {
+    const int yg = ys0 + 4 * g * YG;   // first frame row of this group
+    uint32_t cf[4 * YG];               // this group's CF strip rows
+#pragma unroll
+    for (int r = 0; r < 4 * YG; ++r) cf[r] = load4_clamped(P.cf, P.W, P.H, xs, yg + r);
     const int p = mode_part<MODE>(bx, g * YG);
     const uint32_t mv = __ldg(P.in_mvs + o + p);
-    bvx[g] = 4 * (int)(int16_t)(mv & 0xffffu);
-    bvy[g] = 4 * (int)(int16_t)(mv >> 16);
+    int bvx = 4 * (int)(int16_t)(mv & 0xffffu);
+    int bvy = 4 * (int)(int16_t)(mv >> 16);
+    uint32_t best;
     if (P.in_sads && !SATD) {
-      best[g] = __ldg(P.in_sads + o + p);
+      best = __ldg(P.in_sads + o + p);
     } else {
       uint32_t s = 0;
 #pragma unroll
       for (int j = 0; j < YG; ++j)
-        s += strip_block_dist<SATD>(sf, P.plane, P.pitch, P.pad, xs, ys0 + 4 * (g * YG + j), bvx[g], bvy[g],
-                                    cfs + 4 * (g * YG + j));
-      best[g] = xsum<XMASK>(s);
+        s += strip_block_dist<SATD>(sf, P.plane, P.pitch, P.pad, xs, yg + 4 * j, bvx, bvy, cf + 4 * j);
+      best = xsum<XMASK>(s);
     }
-    if (RD) best[g] += P.lambda * (se_bits(bvx[g]) + se_bits(bvy[g]));   // J at the centre
-  }
-  // ---- half stage ----
-  {
-    int ox[NG], oy[NG];
+    if (RD) best += P.lambda * (se_bits(bvx) + se_bits(bvy));   // J at the centre
+    // ---- half stage ----
+    {
+      const int ox = bvx, oy = bvy;
+      uint32_t sad[8];
+      if (!SATD) {                                    // SAD: one row sweep
+        half_sad_sweep<4 * YG>(sf, P.plane, P.pitch, sf + (size_t)(yg + P.pad) * P.pitch + (xs + P.pad), ox >> 2,
+                               oy >> 2, cf, sad);
+      } else {                                        // SATD: whole 4x4 blocks per candidate
 #pragma unroll
-    for (int g = 0; g < NG; ++g) { ox[g] = bvx[g]; oy[g] = bvy[g]; }
-    uint32_t sad[8][NG];
-    if (!SATD) {                                    // SAD: one row sweep per block group
-      const uint8_t* base = sf + (size_t)(ys0 + P.pad) * P.pitch + (xs + P.pad);
-#pragma unroll
-      for (int g = 0; g < NG; ++g) {
-        uint32_t sg[8];
-        half_sad_sweep<4 * YG>(sf, P.plane, P.pitch, base + (size_t)(4 * g * YG) * P.pitch, ox[g] >> 2, oy[g] >> 2,
-                               cfs + 4 * g * YG, sg);
-#pragma unroll
-        for (int k = 0; k < 8; ++k) sad[k][g] = sg[k];
-      }
-    } else {                                        // SATD: whole 4x4 blocks per candidate
-#pragma unroll
-      for (int k = 0; k < 8; ++k)
-#pragma unroll
-        for (int g = 0; g < NG; ++g) {
+        for (int k = 0; k < 8; ++k) {
           uint32_t t = 0;
 #pragma unroll
           for (int j = 0; j < YG; ++j)
-            t += strip_block_dist<SATD>(sf, P.plane, P.pitch, P.pad, xs, ys0 + 4 * (g * YG + j),
-                                        ox[g] + 2 * c_ring1[k][0], oy[g] + 2 * c_ring1[k][1], cfs + 4 * (g * YG + j));
-          sad[k][g] = t;
+            t += strip_block_dist<SATD>(sf, P.plane, P.pitch, P.pad, xs, yg + 4 * j, ox + 2 * c_ring1[k][0],
+                                        oy + 2 * c_ring1[k][1], cf + 4 * j);
+          sad[k] = t;
         }
-    }
+      }
 #pragma unroll
-    for (int k = 0; k < 8; ++k)
-#pragma unroll
-      for (int g = 0; g < NG; ++g) {
-        const int vx = ox[g] + 2 * c_ring1[k][0], vy = oy[g] + 2 * c_ring1[k][1];
-        uint32_t t = xsum<XMASK>(sad[k][g]);
+      for (int k = 0; k < 8; ++k) {                 // spiral order, strict < (G14)
+        const int vx = ox + 2 * c_ring1[k][0], vy = oy + 2 * c_ring1[k][1];
+        uint32_t t = xsum<XMASK>(sad[k]);
         if (RD) t += P.lambda * (se_bits(vx) + se_bits(vy));
-        if (t < best[g]) { best[g] = t; bvx[g] = vx; bvy[g] = vy; }
+        if (t < best) { best = t; bvx = vx; bvy = vy; }
       }
-  }
-  // ---- quarter stage from the 3x3 half-grid windows around the best half position ----
+    }
+    // ---- quarter stage from the 3x3 half-grid windows around the best half position ----
+    {
+      const int hx = bvx >> 1, hy = bvy >> 1;          // half-grid coordinates (bvx, bvy even)
+      uint32_t qs[8];
+      if (!SATD) {                                     // SAD: one row sweep
+        quarter_sad_sweep<4 * YG>(P.plane, P.pitch, sf + (size_t)(yg + P.pad) * P.pitch + (xs + P.pad), hx, hy, cf, qs);
+      } else {                                         // SATD: whole 4x4 blocks, one candidate at a time
+        const bool mixed = ((hx ^ hy) & 1) != 0;
+        int off[3][3];                                 // window offsets from the strip's row base
 #pragma unroll
-  for (int g = 0; g < NG; ++g) {
-    const int hx = bvx[g] >> 1, hy = bvy[g] >> 1;          // half-grid coordinates (bvx, bvy even)
-    const bool mixed = ((hx ^ hy) & 1) != 0;
-    int off[3][3];                                          // window offsets from the strip's row base
+        for (int b = 0; b < 3; ++b)
 #pragma unroll
-    for (int b = 0; b < 3; ++b)
+          for (int a = 0; a < 3; ++a)
+            off[b][a] = (8 * ((hy + b - 1) & 1) + 2 * ((hx + a - 1) & 1)) * (int)P.plane +
+                        ((hy + b - 1) >> 1) * P.pitch + ((hx + a - 1) >> 1);
 #pragma unroll
-      for (int a = 0; a < 3; ++a)
-        off[b][a] = (8 * ((hy + b - 1) & 1) + 2 * ((hx + a - 1) & 1)) * (int)P.plane +
-                    ((hy + b - 1) >> 1) * P.pitch + ((hx + a - 1) >> 1);
-    uint32_t qs[8];
-#pragma unroll
-    for (int k = 0; k < 8; ++k) qs[k] = 0;
-    const uint8_t* rowp = sf + (size_t)(ys0 + 4 * g * YG + P.pad) * P.pitch + (xs + P.pad);
-    if (!SATD) {                                           // SAD: one row sweep
-      quarter_sad_sweep<4 * YG>(P.plane, P.pitch, sf + (size_t)(ys0 + 4 * g * YG + P.pad) * P.pitch + (xs + P.pad),
-                                hx, hy, cfs + 4 * g * YG, qs);
-    } else {                                               // SATD: whole 4x4 blocks, one candidate at a time
+        for (int k = 0; k < 8; ++k) qs[k] = 0;
+        const uint8_t* rowp = sf + (size_t)(yg + P.pad) * P.pitch + (xs + P.pad);
 #pragma unroll 1
-      for (int jb = 0; jb < YG; ++jb, rowp += 4 * P.pitch) {
-        uint32_t cw[4];
-#pragma unroll
-        for (int r = 0; r < 4; ++r) cw[r] = load4_clamped(P.cf, P.W, P.H, xs, ys0 + 4 * (g * YG + jb) + r);
+        for (int jb = 0; jb < YG; ++jb, rowp += 4 * P.pitch) {
 #pragma unroll 1
-        for (int k = 0; k < 8; ++k) {
-          const int dx = c_ring1[k][0], dy = c_ring1[k][1];
-          // the two half-grid windows this quarter candidate averages (O2 rule, see above)
-          int b0, a0, b1, a1;
-          if (dx == 0 || dy == 0) { b0 = 1; a0 = 1; b1 = 1 + dy; a1 = 1 + dx; }
-          else if (mixed) { b0 = 1; a0 = 1; b1 = 1 + dy; a1 = 1 + dx; }
-          else { b0 = 1; a0 = 1 + dx; b1 = 1 + dy; a1 = 1; }
-          uint32_t smp[4];
+          for (int k = 0; k < 8; ++k) {
+            const int dx = c_ring1[k][0], dy = c_ring1[k][1];
+            // the two half-grid windows this quarter candidate averages (O2 rule, see above)
+            int b0, a0, b1, a1;
+            if (dx == 0 || dy == 0) { b0 = 1; a0 = 1; b1 = 1 + dy; a1 = 1 + dx; }
+            else if (mixed) { b0 = 1; a0 = 1; b1 = 1 + dy; a1 = 1 + dx; }
+            else { b0 = 1; a0 = 1 + dx; b1 = 1 + dy; a1 = 1; }
+            uint32_t smp[4];
 #pragma unroll
-          for (int r = 0; r < 4; ++r) {
-            const uint8_t* rp = rowp + r * P.pitch;
-            const uintptr_t e0 = reinterpret_cast<uintptr_t>(rp + off[b0][a0]);
-            const uintptr_t e1 = reinterpret_cast<uintptr_t>(rp + off[b1][a1]);
-            const uint32_t* w0 = reinterpret_cast<const uint32_t*>(e0 & ~uintptr_t(3));
-            const uint32_t* w1 = reinterpret_cast<const uint32_t*>(e1 & ~uintptr_t(3));
-            smp[r] = vavg4(__funnelshift_r(__ldg(w0), __ldg(w0 + 1), 8u * (uint32_t)(e0 & 3)),
-                           __funnelshift_r(__ldg(w1), __ldg(w1 + 1), 8u * (uint32_t)(e1 & 3)));
+            for (int r = 0; r < 4; ++r) {
+              const uint8_t* rp = rowp + r * P.pitch;
+              const uintptr_t e0 = reinterpret_cast<uintptr_t>(rp + off[b0][a0]);
+              const uintptr_t e1 = reinterpret_cast<uintptr_t>(rp + off[b1][a1]);
+              const uint32_t* w0 = reinterpret_cast<const uint32_t*>(e0 & ~uintptr_t(3));
+              const uint32_t* w1 = reinterpret_cast<const uint32_t*>(e1 & ~uintptr_t(3));
+              smp[r] = vavg4(__funnelshift_r(__ldg(w0), __ldg(w0 + 1), 8u * (uint32_t)(e0 & 3)),
+                             __funnelshift_r(__ldg(w1), __ldg(w1 + 1), 8u * (uint32_t)(e1 & 3)));
+            }
+            qs[k] += satd4(cf + 4 * jb, smp);
           }
-          qs[k] += satd4(cw, smp);
         }
       }
-    }
-    const int ox = bvx[g], oy = bvy[g];
+      const int ox = bvx, oy = bvy;
 #pragma unroll
-    for (int k = 0; k < 8; ++k) {             // spiral order, strict < (G14)
-      const int vx = ox + c_ring1[k][0], vy = oy + c_ring1[k][1];
-      uint32_t t = xsum<XMASK>(qs[k]);
-      if (RD) t += P.lambda * (se_bits(vx) + se_bits(vy));
-      if (t < best[g]) { best[g] = t; bvx[g] = vx; bvy[g] = vy; }
+      for (int k = 0; k < 8; ++k) {             // spiral order, strict < (G14)
+        const int vx = ox + c_ring1[k][0], vy = oy + c_ring1[k][1];
+        uint32_t t = xsum<XMASK>(qs[k]);
+        if (RD) t += P.lambda * (se_bits(vx) + se_bits(vy));
+        if (t < best) { best = t; bvx = vx; bvy = vy; }
+      }
     }
-  }
-  if (writer && (bx & XMASK) == 0) {     // partition leader lane writes
-#pragma unroll
-    for (int g = 0; g < NG; ++g) {
-      const int p = mode_part<MODE>(bx, g * YG);
-      P.out_qmvs[o + p] = (uint32_t)(uint16_t)bvx[g] | ((uint32_t)(uint16_t)bvy[g] << 16);
-      const uint32_t d = best[g] - (RD ? P.lambda * (se_bits(bvx[g]) + se_bits(bvy[g])) : 0);
+    if (writer && (bx & XMASK) == 0) {     // partition leader lane writes
+      P.out_qmvs[o + p] = (uint32_t)(uint16_t)bvx | ((uint32_t)(uint16_t)bvy << 16);
+      const uint32_t d = best - (RD ? P.lambda * (se_bits(bvx) + se_bits(bvy)) : 0);
       P.out_sads[o + p] = (uint16_t)min(d, 65535u);        // SATD can exceed 16 bits (G20)
     }
   }
 }
 
+#ifndef FEVES_SME_MINB
+#define FEVES_SME_MINB 6   // 80 registers, 6 CTAs x 4 warps per SM (measured: 1 -> 243 regs 248 us; 6 -> 183 us; 8 -> 184 us; 10 -> 194 us)
+#endif
 template <bool RD, bool SATD>
-__global__ void __launch_bounds__(128) sme_refine_kernel(const SmeParams P) {
+__global__ void __launch_bounds__(128, FEVES_SME_MINB) sme_refine_kernel(const SmeParams P) {
   const int warp_id = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
   const int n_warps = P.n_rf * P.n_rows * P.groups;
   if (warp_id >= n_warps) return;                    // whole warps exit together
@@ -386,19 +373,16 @@ __global__ void __launch_bounds__(128) sme_refine_kernel(const SmeParams P) {
   const int mbx = min(mbx_raw, P.mb_cols - 1);       // surplus lanes duplicate the last MB
   const int mby = P.row0 + mrow;
   const int xs = 16 * mbx + 4 * bx, ys0 = 16 * mby;
-  uint32_t cfs[16];
-#pragma unroll
-  for (int r = 0; r < 16; ++r) cfs[r] = load4_clamped(P.cf, P.W, P.H, xs, ys0 + r);
   const uint8_t* __restrict__ sf = P.sf[ref];
   const size_t o = ((size_t)(mrow * P.mb_cols + mbx) * P.rf_stride + ref) * kNPart;
   switch (blockIdx.y) {   // one mode per warp: 7x the independent warps (the kernel is latency-bound)
-    case 0: refine_mode<0, 4, 3, RD, SATD>(P, sf, o, bx, xs, ys0, writer, cfs); break;   // 16x16
-    case 1: refine_mode<1, 2, 3, RD, SATD>(P, sf, o, bx, xs, ys0, writer, cfs); break;   // 16x8
-    case 2: refine_mode<2, 4, 1, RD, SATD>(P, sf, o, bx, xs, ys0, writer, cfs); break;   // 8x16
-    case 3: refine_mode<3, 2, 1, RD, SATD>(P, sf, o, bx, xs, ys0, writer, cfs); break;   // 8x8
-    case 4: refine_mode<4, 1, 1, RD, SATD>(P, sf, o, bx, xs, ys0, writer, cfs); break;   // 8x4
-    case 5: refine_mode<5, 2, 0, RD, SATD>(P, sf, o, bx, xs, ys0, writer, cfs); break;   // 4x8
-    default: refine_mode<6, 1, 0, RD, SATD>(P, sf, o, bx, xs, ys0, writer, cfs); break;  // 4x4
+    case 0: refine_mode<0, 4, 3, RD, SATD>(P, sf, o, bx, xs, ys0, writer); break;   // 16x16
+    case 1: refine_mode<1, 2, 3, RD, SATD>(P, sf, o, bx, xs, ys0, writer); break;   // 16x8
+    case 2: refine_mode<2, 4, 1, RD, SATD>(P, sf, o, bx, xs, ys0, writer); break;   // 8x16
+    case 3: refine_mode<3, 2, 1, RD, SATD>(P, sf, o, bx, xs, ys0, writer); break;   // 8x8
+    case 4: refine_mode<4, 1, 1, RD, SATD>(P, sf, o, bx, xs, ys0, writer); break;   // 8x4
+    case 5: refine_mode<5, 2, 0, RD, SATD>(P, sf, o, bx, xs, ys0, writer); break;   // 4x8
+    default: refine_mode<6, 1, 0, RD, SATD>(P, sf, o, bx, xs, ys0, writer); break;  // 4x4
   }
 }
 
