@@ -52,6 +52,9 @@ def parse():
     ap.add_argument("--me-ctas", type=int, default=None, help="ME_OPT_ME_CTAS_PER_SM")
     ap.add_argument("--fused", type=int, default=None, help="ME_OPT_FUSED_SME")
     ap.add_argument("--adaptive", action="store_true", help="N>1: re-split MB rows every frame (SURVEY §8 f3)")
+    ap.add_argument("--exchange", choices=["peer", "collective"], default="peer",
+                    help="N>1: stripe+halo pull and SME stores over peer memory (PeerStream) or NCCL "
+                         "broadcast + gather (ShardedStream; always used with --adaptive)")
     return ap.parse_args()
 
 
@@ -189,7 +192,7 @@ def run_reference(args, cfg):
     v = statistics.mean(vals)
     line = {"impl": "reference", "metric": METRIC, "value": v, "unit": "frames/s", "n_gpus": args.gpus,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 / v, "higher_is_better": True,
-            "scaling": "strong" if args.gpus > 1 else "weak", "vs_baseline": None, "dtype": "u8",
+            "scaling": "strong", "vs_baseline": None, "dtype": "u8",
             "data": "synthetic (gen-tex, seeded)", "config": config_json(cfg, args),
             "cpu_baseline": {"kind": cb["kind"], "cores": cb["cores"], "sample": cb["sample"], "value": v,
                              "unit": "frames/s"},
@@ -201,7 +204,8 @@ def run_reference(args, cfg):
 def config_json(cfg, args):
     return {"workload": cfg.name, "baseline_config_index": cfg.baseline_index, "width": cfg.width,
             "height": cfg.height, "n_rf": cfg.n_rf, "sa_range": cfg.sa_range, "path": "int+me+sme (IPPP stream)",
-            "partitions": 41, "parallelism": f"mb-row x{args.gpus}" + (" adaptive" if args.adaptive else ""),
+            "partitions": 41, "parallelism": f"mb-row x{args.gpus}" + (" adaptive" if args.adaptive else "") +
+            (f" ({args.exchange} exchange)" if args.gpus > 1 and not args.adaptive else ""),
             "l2": "flushed (512 MiB write) before every timed step"}
 
 
@@ -225,7 +229,7 @@ def run_feves(args, cfg):
     import __graft_entry__ as ge
     ge.build()
     import paper_conf_icpp_ilicmrs14_b200 as feves
-    from paper_conf_icpp_ilicmrs14_b200.shard import ShardedStream, stripes
+    from paper_conf_icpp_ilicmrs14_b200.shard import PeerStream, ShardedStream, stripes
     from synth import ippp_sequence
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
@@ -256,7 +260,13 @@ def run_feves(args, cfg):
     pinned = [torch.from_numpy(f).pin_memory() for f in host]
     buf = torch.empty_like(frames[0])
     flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
-    ss = ShardedStream(me, adaptive=args.adaptive) if world > 1 else None
+    peer = world > 1 and args.exchange == "peer" and not args.adaptive
+    if world == 1:
+        ss = None
+    elif peer:
+        ss = PeerStream(me)
+    else:
+        ss = ShardedStream(me, adaptive=args.adaptive)
 
     def push(t):
         if ss is not None:
@@ -343,8 +353,9 @@ def run_feves(args, cfg):
     # ---- e2e: pinned host frame in, host MVs/SADs out, every step ----
     e2e = None
     if not args.no_e2e and world > 1:
-        # sharded: rank 0 uploads the pinned frame, broadcast + per-rank push + gather
-        # (ShardedStream), rank 0 downloads the assembled quarter-pel MVs + SADs
+        # sharded: rank 0 uploads the pinned frame, the ranks exchange stripes (PeerStream:
+        # peer memory; ShardedStream: broadcast + gather), rank 0 downloads the assembled
+        # quarter-pel MVs + SADs
         me.stream_reset()
         for i in range(cfg.n_rf + 2):
             ss.push(frames[i % n_frames], buf)
@@ -355,9 +366,12 @@ def run_feves(args, cfg):
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record(stream)
         for i in range(args.e2e_steps):
-            if rank == 0:
+            if rank == 0 and not peer:
                 buf.copy_(pinned[(cfg.n_rf + 2 + i) % n_frames], non_blocking=True)
-            r = ss.push(buf, buf)
+            if peer:
+                r = ss.push(pinned[(cfg.n_rf + 2 + i) % n_frames] if rank == 0 else None)
+            else:
+                r = ss.push(buf, buf)
             if rank == 0:
                 qm_h.copy_(r[0], non_blocking=True)
                 qs_h.copy_(r[1], non_blocking=True)
@@ -368,8 +382,11 @@ def run_feves(args, cfg):
         e2e = {"value": args.e2e_steps / (float(tt.item()) / 1e3), "unit": "frames/s",
                "h2d_bytes_per_step": pinned[0].numel(),
                "d2h_bytes_per_step": qm_h.numel() * 2 + qs_h.numel() * 2,
-               "api": "ShardedStream.push (NCCL broadcast in, per-rank me_stream_push, NCCL gather out), "
-                      "pinned buffers on rank 0"}
+               "api": ("PeerStream.push (rank 0 uploads the pinned frame; each rank pulls its stripe + halo "
+                       "rows over peer memory and its SME stores into rank 0's buffer; two 4-byte NCCL "
+                       "all-reduces per frame)" if peer else
+                       "ShardedStream.push (NCCL broadcast in, per-rank me_stream_push, NCCL gather out)")
+                      + ", pinned buffers on rank 0"}
     if not args.no_e2e and world == 1:
         qm_h = torch.empty(me.mv_shape() + (2,), dtype=torch.int16).pin_memory()
         qs_h = torch.empty(me.mv_shape(), dtype=torch.uint16).pin_memory()
@@ -400,7 +417,7 @@ def run_feves(args, cfg):
     line = {
         "metric": METRIC, "value": fps, "unit": "frames/s", "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": total_ms / args.steps, "higher_is_better": True,
-        "scaling": "strong" if world > 1 else "weak", "vs_baseline": None, "dtype": "u8",
+        "scaling": "strong", "vs_baseline": None, "dtype": "u8",
         "data": "synthetic (gen-tex: 8 sinusoids in (1.25,-0.75) px/frame motion + noise, seeded)",
         "config": config_json(cfg, args),
         "candidate_gsad_per_s": u["gsad"] * fps / 1e9,

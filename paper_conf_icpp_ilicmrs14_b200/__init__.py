@@ -61,9 +61,13 @@ def lib():
         L.me_set_fused.argtypes = [P, i]
         L.me_set_option.argtypes = [P, i, i]
         L.me_mode_decision.argtypes = [P, P, P, P]
+        L.me_ipc_export.argtypes = [P, P, P, ctypes.POINTER(ctypes.c_size_t)]
+        L.me_ipc_open.argtypes = [P, P, ctypes.c_size_t, ctypes.c_size_t, ctypes.POINTER(ctypes.c_void_p)]
+        L.me_ipc_close.argtypes = [P, P]
         for fn in ("me_set_stream", "me_set_rows", "me_get_layout", "me_estimate", "int_interpolate",
                    "sme_refine", "me_encode_frame", "me_last_launch_count", "me_stream_reset",
-                   "me_stream_push", "me_stream_outputs", "me_sync", "me_set_timing", "me_get_timings", "me_set_fused", "me_set_option", "me_mode_decision"):
+                   "me_stream_push", "me_stream_outputs", "me_sync", "me_set_timing", "me_get_timings", "me_set_fused", "me_set_option", "me_mode_decision",
+                   "me_ipc_export", "me_ipc_open", "me_ipc_close"):
             getattr(L, fn).restype = i
         _lib = L
     return _lib
@@ -205,8 +209,36 @@ class MotionEstimator:
                                     int(out_host), ctypes.byref(n)))
         return qmvs, qsads, n.value
 
+    def stream_push_ptr(self, cf_ptr: int, qmvs_ptr: int, qsads_ptr: int, bind_stream=True):
+        """me_stream_push on raw device addresses (e.g. peer buffers mapped by
+        ``ipc_open``): frame t read from ``cf_ptr``, this stripe's quarter-pel MVs /
+        SADs written at ``qmvs_ptr`` / ``qsads_ptr``.  Returns n_ref_used."""
+        n = ctypes.c_int()
+        if bind_stream:
+            self._bind_stream()
+        _check(lib().me_stream_push(self._ctx, cf_ptr, 0, qmvs_ptr, qsads_ptr, 0, ctypes.byref(n)))
+        return n.value
+
     def sync(self):
         _check(lib().me_sync(self._ctx))
+
+    # ------------------------------------------------- peer memory (8e) --
+    def ipc_export(self, t):
+        """(64-byte CUDA IPC handle, byte offset) of device tensor ``t`` (me_ipc_export)."""
+        h = ctypes.create_string_buffer(64)
+        off = ctypes.c_size_t()
+        _check(lib().me_ipc_export(self._ctx, t.data_ptr(), h, ctypes.byref(off)))
+        return h.raw, off.value
+
+    def ipc_open(self, handle: bytes, offset: int, nbytes: int) -> int:
+        """Map another process's exported buffer; returns its device address (me_ipc_open)."""
+        p = ctypes.c_void_p()
+        _check(lib().me_ipc_open(self._ctx, ctypes.create_string_buffer(handle, 64), offset, nbytes,
+                                 ctypes.byref(p)))
+        return p.value
+
+    def ipc_close(self, ptr: int):
+        _check(lib().me_ipc_close(self._ctx, ptr))
 
     # ---------------------------------------------- module timers (P:87) --
     def set_fused(self, on: bool = True):
@@ -214,6 +246,7 @@ class MotionEstimator:
         _check(lib().me_set_fused(self._ctx, int(on)))
 
     OPT_FUSED_SME, OPT_PIPELINE_RF, OPT_ME_CTAS_PER_SM, OPT_LAMBDA, OPT_SME_SATD, OPT_SA_INCLUSIVE = 1, 2, 3, 4, 5, 6
+    OPT_HALO_ONLY = 7
 
     def set_sa_inclusive(self, on: bool = True):
         """Candidates in [-S/2, +S/2]^2 (G1 alternative reading, f4)."""

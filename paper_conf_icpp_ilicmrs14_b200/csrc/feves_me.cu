@@ -6,6 +6,8 @@
 // me_encode_frame, and its stream.  No allocation on the per-frame path.
 #include "../../include/feves_me.h"
 
+#include <cuda.h>   // CUdeviceptr / CUresult types only: driver calls go through cudaGetDriverEntryPoint
+
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
@@ -68,6 +70,10 @@ struct me_ctx {
   cudaStream_t sme_st;   // pipeline: SME stream
   cudaEvent_t ev_me[kMaxRf], ev_sme_done;
   int sf_v0[kMaxRf], sf_v1[kMaxRf];   // MB rows whose SF rows each SF-ring slot holds (re-split support)
+  int halo_only;                      // ME_OPT_HALO_ONLY: pushes copy the stripe + halo rows only
+  int fv0[kMaxRf + 2], fv1[kMaxRf + 2];   // frame rows each frame-ring slot holds
+  struct Peer { uintptr_t lo, hi; void* base; } peers[16];   // me_ipc_open mappings
+  int n_peers;
 };
 
 static thread_local int g_last_error = ME_OK;
@@ -82,8 +88,17 @@ static int spiral_rank_closed_form(int dx, int dy) {   // G4
   return base + 2 * (2 * l - 1) + 2 * (dy + l) + (dx > 0 ? 1 : 0);
 }
 
+static bool is_peer_ptr(const me_ctx* c, const void* p) {
+  for (int i = 0; i < c->n_peers; ++i)
+    if (c->peers[i].base && reinterpret_cast<uintptr_t>(p) >= c->peers[i].lo &&
+        reinterpret_cast<uintptr_t>(p) < c->peers[i].hi)
+      return true;
+  return false;
+}
+
 static bool is_device_ptr(me_ctx* c, const void* p) {
   if (!p) return false;
+  if (is_peer_ptr(c, p)) return true;   // peer memory mapped by me_ipc_open (another GPU's buffer)
   for (int i = 0; i < c->n_checked; ++i)
     if (c->checked[i] == p) return true;
   cudaPointerAttributes a;
@@ -217,6 +232,8 @@ extern "C" void me_destroy(me_ctx* c) {
   if (c->ev_fork) cudaEventDestroy(c->ev_fork);
   if (c->ev_join) cudaEventDestroy(c->ev_join);
   if (c->own_stream && c->stream) cudaStreamDestroy(c->stream);
+  for (int i = 0; i < c->n_peers; ++i)
+    if (c->peers[i].base) cudaIpcCloseMemHandle(c->peers[i].base);
   delete c;
 }
 
@@ -362,6 +379,7 @@ static int launch_sme(me_ctx* c, const uint8_t* cf, const uint8_t* const* sfs, c
   P.lambda = c->lambda;
   P.pad = c->sf_pad; P.pitch = c->sf_pitch;
   P.plane = (size_t)c->sf_rows * c->sf_pitch;
+  P.fence = is_peer_ptr(c, out_qmvs) || is_peer_ptr(c, out_sads);
   const int warps = n_ref * P.n_rows * P.groups;
   tmark(c, 4, st);
   const dim3 sg((warps + 3) / 4, 7);   // y = partition mode
@@ -530,17 +548,30 @@ extern "C" int me_stream_push(me_ctx* c, const uint8_t* cf, int cf_on_host, int1
   const long long t = c->t;
   const int par = (int)(t & 1);
   uint8_t* cur = c->ring + (size_t)(t % slots) * fb;
+  // rows of every frame this stripe reads (ME +-R, SME +1, 6-tap -2..+3)
+  int y0 = 0, y1 = c->H;
+  if (c->halo_only) {
+    y0 = std::max(0, 16 * c->row0 - c->R - 6);
+    y1 = std::min(c->H, 16 * c->row1 + c->R + 7);
+  }
+  const int n_ref = (int)std::min<long long>(t, c->n_rf);
+  for (int k = 0; k < n_ref; ++k) {             // a re-split may need rows a halo-only frame lacks
+    const int s = (int)((t - 1 - k) % slots);
+    if (c->fv0[s] > y0 || c->fv1[s] < y1) return ME_ESTATE;
+  }
+  const size_t off = (size_t)y0 * c->W, len = (size_t)(y1 - y0) * c->W;
   if (cf_on_host) {
     // upload on the copy-in stream once the compute of push t-2 (last reader of this slot) is done
     if (cudaStreamWaitEvent(c->copy_in, c->ev_done[par], 0) != cudaSuccess ||
-        cudaMemcpyAsync(cur, cf, fb, cudaMemcpyHostToDevice, c->copy_in) != cudaSuccess ||
+        cudaMemcpyAsync(cur + off, cf + off, len, cudaMemcpyHostToDevice, c->copy_in) != cudaSuccess ||
         cudaEventRecord(c->ev_up[par], c->copy_in) != cudaSuccess ||
         cudaStreamWaitEvent(c->stream, c->ev_up[par], 0) != cudaSuccess)
       return launch_status();
-  } else if (cudaMemcpyAsync(cur, cf, fb, cudaMemcpyDeviceToDevice, c->stream) != cudaSuccess) {
-    return launch_status();
+  } else if (cudaMemcpyAsync(cur + off, cf + off, len, cudaMemcpyDefault, c->stream) != cudaSuccess) {
+    return launch_status();   // (cudaMemcpyDefault: cf may be a peer GPU's buffer, me_ipc_open)
   }
-  const int n_ref = (int)std::min<long long>(t, c->n_rf);
+  c->fv0[t % slots] = y0;
+  c->fv1[t % slots] = y1;
   if (n_ref_used) *n_ref_used = n_ref;
   if (n_ref > 0) {
     uint8_t* new_rf = c->ring + (size_t)((t - 1) % slots) * fb;
@@ -655,6 +686,9 @@ extern "C" int me_set_option(me_ctx* c, int option, int value) {
     case ME_OPT_SME_SATD:
       c->satd = value ? 1 : 0;
       return ME_OK;
+    case ME_OPT_HALO_ONLY:
+      c->halo_only = value ? 1 : 0;
+      return ME_OK;
     case ME_OPT_LAMBDA:
       if (value < 0 || value > 2000) return ME_EINVAL;
       if (c->stream) cudaStreamSynchronize(c->stream);   // the table may be in use
@@ -662,6 +696,90 @@ extern "C" int me_set_option(me_ctx* c, int option, int value) {
       return upload_key_table(c);
     default: return ME_EINVAL;
   }
+}
+
+// ------------------------------------------------------------ peer memory ----
+// stripe inputs and outputs move over NVLink by loads/stores of the
+// kernels and copy engines instead of broadcast/gather collectives.
+static int alloc_base(const void* p, uintptr_t* base) {
+  using AddrRange = CUresult (*)(CUdeviceptr*, size_t*, CUdeviceptr);
+  static AddrRange fn = nullptr;
+  if (!fn) {
+    void* f = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuMemGetAddressRange", &f, cudaEnableDefault, &q) != cudaSuccess || !f ||
+        q != cudaDriverEntryPointSuccess) {
+      cudaGetLastError();
+      return ME_ECUDA;
+    }
+    fn = reinterpret_cast<AddrRange>(f);
+  }
+  CUdeviceptr b = 0;
+  size_t sz = 0;
+  if (fn(&b, &sz, reinterpret_cast<CUdeviceptr>(p)) != CUDA_SUCCESS) return ME_EINVAL;
+  *base = static_cast<uintptr_t>(b);
+  return ME_OK;
+}
+
+extern "C" int me_ipc_export(me_ctx* c, const void* dptr, void* handle, size_t* offset) {
+  if (!c || !handle || !offset || !is_device_ptr(c, dptr)) return ME_EINVAL;
+  for (int i = 0; i < c->n_peers; ++i)   // only this device's own allocations can be exported
+    if (reinterpret_cast<uintptr_t>(dptr) >= c->peers[i].lo && reinterpret_cast<uintptr_t>(dptr) < c->peers[i].hi)
+      return ME_EINVAL;
+  uintptr_t base = 0;
+  int st = alloc_base(dptr, &base);
+  if (st != ME_OK) return st;
+  cudaIpcMemHandle_t h;
+  if (cudaIpcGetMemHandle(&h, reinterpret_cast<void*>(base)) != cudaSuccess) {
+    cudaGetLastError();
+    return ME_ECUDA;
+  }
+  static_assert(sizeof(h) == ME_IPC_HANDLE_BYTES, "CUDA IPC handle size");
+  std::memcpy(handle, &h, sizeof(h));
+  *offset = reinterpret_cast<uintptr_t>(dptr) - base;
+  return ME_OK;
+}
+
+extern "C" int me_ipc_open(me_ctx* c, const void* handle, size_t offset, size_t bytes, void** dptr) {
+  if (!c || !handle || !dptr || bytes == 0) return ME_EINVAL;
+  int slot = -1;
+  for (int i = 0; i < c->n_peers; ++i)
+    if (!c->peers[i].base) { slot = i; break; }
+  if (slot < 0) {
+    if (c->n_peers == 16) return ME_EINVAL;
+    slot = c->n_peers++;
+  }
+  cudaIpcMemHandle_t h;
+  std::memcpy(&h, handle, sizeof(h));
+  int dev = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess || (dev != c->device && cudaSetDevice(c->device) != cudaSuccess)) {
+    cudaGetLastError();
+    return ME_ECUDA;
+  }
+  void* base = nullptr;
+  const cudaError_t e = cudaIpcOpenMemHandle(&base, h, cudaIpcMemLazyEnablePeerAccess);
+  if (dev != c->device) cudaSetDevice(dev);
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    return e == cudaErrorInvalidValue || e == cudaErrorInvalidResourceHandle ? ME_EINVAL : ME_ECUDA;
+  }
+  const uintptr_t lo = reinterpret_cast<uintptr_t>(base) + offset;
+  c->peers[slot] = {lo, lo + bytes, base};
+  *dptr = reinterpret_cast<void*>(lo);
+  return ME_OK;
+}
+
+extern "C" int me_ipc_close(me_ctx* c, void* dptr) {
+  if (!c || !dptr) return ME_EINVAL;
+  for (int i = 0; i < c->n_peers; ++i)
+    if (c->peers[i].base && c->peers[i].lo == reinterpret_cast<uintptr_t>(dptr)) {
+      if (c->stream) cudaStreamSynchronize(c->stream);   // kernels may still use it
+      const cudaError_t e = cudaIpcCloseMemHandle(c->peers[i].base);
+      c->peers[i] = {0, 0, nullptr};
+      c->n_checked = 0;                                 // drop cached pointer checks
+      return e == cudaSuccess ? ME_OK : ME_ECUDA;
+    }
+  return ME_EINVAL;
 }
 
 extern "C" int me_set_fused(me_ctx* c, int on) { return me_set_option(c, ME_OPT_FUSED_SME, on); }

@@ -35,6 +35,7 @@ struct SmeParams {
   int pad, pitch;
   size_t plane;
   int lambda;                                         // G18 rate term (0 = pure SAD, G13)
+  int fence;                                          // outputs are peer memory (me_ipc_open): system fence at exit
 };
 
 // ring-1 spiral order s_k (G12/G14), compile-time so unrolled loops fold it
@@ -384,6 +385,7 @@ __global__ void __launch_bounds__(128, FEVES_SME_MINB) sme_refine_kernel(const S
     case 5: refine_mode<5, 2, 0, RD, SATD>(P, sf, o, bx, xs, ys0, writer); break;   // 4x8
     default: refine_mode<6, 1, 0, RD, SATD>(P, sf, o, bx, xs, ys0, writer); break;  // 4x4
   }
+  if (P.fence) __threadfence_system();   // stores to another GPU's buffer are performed before the kernel ends
 }
 
 }  // namespace feves

@@ -179,3 +179,91 @@ class ShardedStream:
             return torch.cat(parts_m).to(dev), torch.cat(parts_s).to(dev), n_ref
         dist.gather(payload, None, dst=self.src, group=self.group)
         return None
+
+
+class PeerStream:
+    """IPPP stream over G ranks with the exchange done in peer memory (SURVEY §8(e),
+    "Option to fuse the collective"; BJ north_star "reference-frame rows plus an
+    SA-radius halo via ... P2P over NVLink").
+
+    Rank ``src`` owns two frame slots and two full-frame output buffers and exports
+    them (``me_ipc_export``); every other rank maps them (``me_ipc_open``).  Per frame t:
+      1. rank src copies frame t into slot t mod 2;
+      2. barrier #1 (stream-ordered: a 4-byte NCCL all-reduce, no host sync);
+      3. every rank runs ``me_stream_push`` with the frame read from rank src's slot
+         (``ME_OPT_HALO_ONLY``: the copy engine pulls only the stripe + halo rows,
+         [16 r0 - R - 6, 16 r1 + R + 7), over NVLink) and with the outputs pointed at
+         its stripe's rows of rank src's output buffer t mod 2: the SME kernel's
+         stores travel over NVLink, so there is no gather collective and no copy;
+      4. barrier #2: every stripe of frame t is in rank src's buffer.
+    Slot reuse is safe: rank src overwrites slot t mod 2 at frame t+2, after barrier
+    #2 of frame t+1, which every rank passes only after its push of frame t has read
+    that slot.  The tensors returned on rank src stay valid until push t+2.
+    Results equal the single-GPU stream bitwise (pin P11); the split is the static
+    equidistant one -- with the adaptive re-split use ``ShardedStream``.
+    Over gloo (one shared GPU in tests) the barriers synchronise the host instead."""
+
+    def __init__(self, me, group=None, src: int = 0):
+        self.me, self.group, self.src = me, group, src
+        self.rank = dist.get_rank(group)
+        self.world = dist.get_world_size(group)
+        self.nccl = dist.get_backend(group) == "nccl"
+        self.cur = stripes(me.mb_rows, self.world)
+        r0, r1 = self.cur[self.rank]
+        me.set_rows(r0, r1)
+        me.set_option(me.OPT_HALO_ONLY, 1)
+        dev = me.device
+        H, W = me.height, me.width
+        shape = (me.mb_rows, me.mb_cols, me.n_rf, 41)
+        self.row_bytes = (me.mb_cols * me.n_rf * 41 * 4, me.mb_cols * me.n_rf * 41 * 2)
+        if self.rank == src:
+            self.frames = [torch.empty((H, W), dtype=torch.uint8, device=dev) for _ in range(2)]
+            self.qm = [torch.empty(shape + (2,), dtype=torch.int16, device=dev) for _ in range(2)]
+            self.qs = [torch.empty(shape, dtype=torch.uint16, device=dev) for _ in range(2)]
+            bufs = self.frames + self.qm + self.qs
+            exported = [me.ipc_export(b) + (b.numel() * b.element_size(),) for b in bufs]
+        else:
+            exported = None
+        allx = [None] * self.world
+        dist.all_gather_object(allx, exported, group=group)
+        if self.rank == src:
+            ptrs = [b.data_ptr() for b in bufs]
+            self.opened = []
+        else:
+            ptrs = [me.ipc_open(h, off, n) for h, off, n in allx[src]]
+            self.opened = list(ptrs)
+        self.f_ptr, self.qm_ptr, self.qs_ptr = ptrs[0:2], ptrs[2:4], ptrs[4:6]
+        self.flag = torch.zeros(1, dtype=torch.int32, device=dev if self.nccl else "cpu")
+        self.t = 0
+
+    def _barrier(self):
+        if self.nccl:
+            dist.all_reduce(self.flag, group=self.group)   # ordered on the current stream
+        else:
+            torch.cuda.current_stream(self.me.device).synchronize()
+            dist.barrier(group=self.group)
+
+    def push(self, frame, frame_buf=None):
+        """frame: this step's frame on rank ``src`` (device or pinned host tensor [H, W]);
+        ignored elsewhere.  Returns (qmvs, qsads, n_ref) of the WHOLE frame on rank src,
+        None elsewhere."""
+        b = self.t & 1
+        if self.rank == self.src:
+            self.frames[b].copy_(frame.view(self.me.height, self.me.width), non_blocking=True)
+        self._barrier()
+        r0 = self.cur[self.rank][0]
+        n_ref = self.me.stream_push_ptr(self.f_ptr[b], self.qm_ptr[b] + r0 * self.row_bytes[0],
+                                        self.qs_ptr[b] + r0 * self.row_bytes[1])
+        self._barrier()
+        self.t += 1
+        if self.rank == self.src:
+            return self.qm[b], self.qs[b], n_ref
+        return None
+
+    def close(self):
+        """Unmap rank src's buffers (collective: rank src keeps them alive until all closed)."""
+        self.me.sync()
+        for p in self.opened:
+            self.me.ipc_close(p)
+        self.opened = []
+        dist.barrier(group=self.group)

@@ -76,3 +76,76 @@ def test_two_rank_sharded_stream_equals_single(adaptive):
     assert ok
     if adaptive:                       # rank 1 reported 3x the time per row: rows moved to rank 0
         assert history[0] == [(0, 4), (4, 8)] and history[-1] == [(0, 6), (6, 8)]
+
+
+def _peer_worker(rank, world, port, q, host_frames):
+    import torch.distributed as dist
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        import paper_conf_icpp_ilicmrs14_b200 as F
+        from paper_conf_icpp_ilicmrs14_b200.shard import PeerStream
+        from synth import gen_tex
+        torch.cuda.set_device(0)
+        me = F.MotionEstimator(W, H, S, N_RF)
+        ps = PeerStream(me)
+        frames = [torch.from_numpy(gen_tex(W, H, t, 37)) for t in range(N_FRAMES)]
+        frames = [f.pin_memory() if host_frames else f.cuda() for f in frames]
+        outs = []
+        for t in range(N_FRAMES):
+            r = ps.push(frames[t] if rank == 0 else None)
+            if rank == 0:
+                outs.append((r[0].cpu().numpy(), r[1].cpu().numpy(), r[2]))
+        ps.close()
+        if rank == 0:
+            ref = F.MotionEstimator(W, H, S, N_RF)
+            refs = []
+            for t in range(N_FRAMES):
+                qm, qs, n = ref.stream_push(frames[t].cuda())
+                refs.append((qm.cpu().numpy(), qs.cpu().numpy(), n))
+            ok = all(np.array_equal(a[0][:, :, :a[2]], b[0][:, :, :b[2]]) and
+                     np.array_equal(a[1][:, :, :a[2]], b[1][:, :, :b[2]]) and a[2] == b[2]
+                     for a, b in zip(outs, refs))
+            q.put(ok)
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world,host_frames", [(2, False), (3, True)])
+def test_peer_stream_equals_single(world, host_frames):
+    """PeerStream (SURVEY §8(e) fused exchange): frames pulled as stripe + halo rows from
+    rank 0's IPC-exported slot, SME outputs stored straight into rank 0's IPC-exported
+    buffer (no broadcast/gather) == one full-frame stream, bitwise.  The ranks share
+    cuda:0 here (same-device CUDA IPC); on the 8-GPU box the same stores cross NVLink."""
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    with socket.socket() as s:
+        s.bind(("127.0.0.1", 0))
+        port = s.getsockname()[1]
+    procs = [ctx.Process(target=_peer_worker, args=(r, world, port, q, host_frames)) for r in range(world)]
+    for p in procs:
+        p.start()
+    ok = q.get(timeout=600)
+    for p in procs:
+        p.join(timeout=120)
+        assert p.exitcode == 0
+    assert ok
+
+
+def test_halo_only_push_refuses_missing_rows():
+    """ME_OPT_HALO_ONLY copies only the stripe + halo rows; a later push whose stripe
+    needs rows an older ring frame lacks must fail with ME_ESTATE, not read garbage."""
+    import paper_conf_icpp_ilicmrs14_b200 as F
+    from synth import gen_tex
+    me = F.MotionEstimator(W, H, S, N_RF)
+    me.set_rows(0, 2)
+    me.set_option(me.OPT_HALO_ONLY, 1)
+    frames = [torch.from_numpy(gen_tex(W, H, t, 41)).cuda() for t in range(3)]
+    me.stream_push(frames[0])
+    me.stream_push(frames[1])
+    me.set_rows(6, 8)                   # rows 96..119 were never copied for frames 0, 1
+    with pytest.raises(F.FevesError, match="state"):
+        me.stream_push(frames[2])
+    me.set_rows(0, 2)                   # the original stripe still works
+    me.stream_push(frames[2])
+    torch.cuda.synchronize()
