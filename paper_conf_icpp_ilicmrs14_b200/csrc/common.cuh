@@ -18,13 +18,25 @@ __device__ __forceinline__ uint32_t vad4(uint32_t a, uint32_t b, uint32_t c) {
 }
 
 // per-byte rounded average (u+v+1)>>1 on 4 packed bytes.  PTX vavrg4 is NOT
-// native on sm_100a (ptxas expands it byte by byte, ~16 instructions), so use
-// the exact SWAR identity ceil((a+b)/2) = (a|b) - ((a^b)>>1) per byte; the mask
-// stops bit 0 of a byte from shifting into its neighbour, and the subtraction
-// never borrows across bytes because (a^b)>>1 <= a|b bytewise.  4 ALU ops.
-__device__ __forceinline__ uint32_t vavg4(uint32_t a, uint32_t b) {
-  return (a | b) - (((a ^ b) & 0xfefefefeu) >> 1);
+// native on sm_100a (ptxas expands it byte by byte, ~16 instructions).  Exact
+// SWAR form: ceil((a+b)/2) = y + (x >> 1) per byte with
+//   y = (a & b) | ((a ^ b) & 0x01)   (= floor part + carry-in bit; ONE LOP3),
+//   x = (a ^ b) & 0xfe               (ONE LOP3; bit 0 of every byte cleared, so
+//                                     the 32-bit shift moves nothing across bytes),
+// and y + (x >> 1) = hi32(x * 2^31) + y as ONE IMAD.HI on the FMA pipe (the
+// per-byte sum is the average <= 255, so no carry crosses a byte).  k_hi must be
+// 0x80000000 supplied at run time (a kernel parameter): a literal would be
+// strength-reduced by ptxas into SHF + IADD on the ALU pipe, which is the pipe
+// INT and SME are bound by.  2 ALU + 1 FMA instead of 4 ALU + 1 FMA.
+// (Checked exhaustively over all byte pairs on the host; parity tests.)
+__device__ __forceinline__ uint32_t vavg4(uint32_t a, uint32_t b, uint32_t k_hi) {
+  const uint32_t y = (a & b) | ((a ^ b) & 0x01010101u);
+  const uint32_t x = (a ^ b) & 0xfefefefeu;
+  uint32_t d;
+  asm("mad.hi.u32 %0, %1, %2, %3;" : "=r"(d) : "r"(x), "r"(k_hi), "r"(y));
+  return d;
 }
+constexpr uint32_t kAvgHi = 0x80000000u;   // the run-time k_hi of vavg4 (host side)
 
 __device__ __forceinline__ int clampi(int v, int lo, int hi) { return v < lo ? lo : (v > hi ? hi : v); }
 

@@ -333,6 +333,7 @@ static int launch_me(me_ctx* c, const uint8_t* cf, const uint8_t* const* rfs, in
 static int launch_int(me_ctx* c, const uint8_t* rf, uint8_t* sf, cudaStream_t st) {
   IntParams P;
   P.rf = rf; P.sf = sf; P.W = c->W; P.H = c->H;
+  P.k_hi = kAvgHi;
   P.pad = c->sf_pad; P.pitch = c->sf_pitch; P.rows = c->sf_rows;
   P.plane = (size_t)c->sf_rows * c->sf_pitch;
   if (c->row0 == 0 && c->row1 == c->mb_rows) {
@@ -380,6 +381,7 @@ static int launch_sme(me_ctx* c, const uint8_t* cf, const uint8_t* const* sfs, c
   P.pad = c->sf_pad; P.pitch = c->sf_pitch;
   P.plane = (size_t)c->sf_rows * c->sf_pitch;
   P.fence = is_peer_ptr(c, out_qmvs) || is_peer_ptr(c, out_sads);
+  P.k_hi = kAvgHi;
   const int warps = n_ref * P.n_rows * P.groups;
   tmark(c, 4, st);
   const dim3 sg((warps + 3) / 4, 7);   // y = partition mode

@@ -11,7 +11,7 @@
 // One thread = 16 consecutive plane columns of one plane row.  The 6-tap
 // filters on b1/h1/s1 (range [-2550, 10710]) run two columns per 32-bit
 // instruction on biased, non-negative 16-bit lanes (plain IADD / IMAD by 20
-// and -5, exact per lane); j1 (20-bit) runs in int32.  Quarter samples: VAVRG4 on 4 packed
+// and -5, exact per lane); j1 (20-bit) runs in int32.  Quarter samples: SWAR vavg4 on 4 packed
 // bytes.  A warp writes 32 x 16 B = 512 contiguous bytes per plane with
 // 128-bit stores (HBM-bound kernel: 1 B read + 16 B written per position).
 #pragma once
@@ -26,6 +26,7 @@ struct IntParams {
   size_t plane;   // bytes per phase plane = rows * pitch
   int g_lo, g_hi; // interior 16-column groups [g_lo, g_hi): every source word in-frame and aligned
   int border_bx;  // border blocks: groups per block row (power of two >= number of border groups)
+  uint32_t k_hi;  // = kAvgHi (vavg4)
 };
 
 // Two columns per 32-bit register, one per 16-bit lane, and every lane kept
@@ -131,27 +132,28 @@ __device__ __forceinline__ void int_body(const IntParams& P, int g, int rr) {
                         0x5410);
   }
 
+  const uint32_t kh = P.k_hi;
   uint8_t* dst = P.sf + (size_t)rr * P.pitch + 16 * g;
   auto put = [&](int ph, uint32_t a, uint32_t b, uint32_t c, uint32_t d) {
     *reinterpret_cast<uint4*>(dst + ph * P.plane) = make_uint4(a, b, c, d);
   };
 #define PLANE(ph, EXPR) put(ph, EXPR(0), EXPR(1), EXPR(2), EXPR(3))
 #define G_(q) Gw[q]
-#define A_(q) vavg4(Gw[q], bw[q])
+#define A_(q) vavg4(Gw[q], bw[q], kh)
 #define B_(q) bw[q]
-#define C_(q) vavg4(Hw[q], bw[q])
-#define D_(q) vavg4(Gw[q], hw[q])
-#define E_(q) vavg4(bw[q], hw[q])
-#define F_(q) vavg4(bw[q], jw[q])
-#define Gq_(q) vavg4(bw[q], mw[q])
+#define C_(q) vavg4(Hw[q], bw[q], kh)
+#define D_(q) vavg4(Gw[q], hw[q], kh)
+#define E_(q) vavg4(bw[q], hw[q], kh)
+#define F_(q) vavg4(bw[q], jw[q], kh)
+#define Gq_(q) vavg4(bw[q], mw[q], kh)
 #define H_(q) hw[q]
-#define I_(q) vavg4(hw[q], jw[q])
+#define I_(q) vavg4(hw[q], jw[q], kh)
 #define J_(q) jw[q]
-#define K_(q) vavg4(jw[q], mw[q])
-#define N_(q) vavg4(Mw[q], hw[q])
-#define Pq_(q) vavg4(hw[q], sw[q])
-#define Q_(q) vavg4(jw[q], sw[q])
-#define R_(q) vavg4(mw[q], sw[q])
+#define K_(q) vavg4(jw[q], mw[q], kh)
+#define N_(q) vavg4(Mw[q], hw[q], kh)
+#define Pq_(q) vavg4(hw[q], sw[q], kh)
+#define Q_(q) vavg4(jw[q], sw[q], kh)
+#define R_(q) vavg4(mw[q], sw[q], kh)
   // phase = 4*yFrac + xFrac (G11); names as in DESIGN.md O2
   PLANE(0, G_);  PLANE(1, A_);  PLANE(2, B_);   PLANE(3, C_);
   PLANE(4, D_);  PLANE(5, E_);  PLANE(6, F_);   PLANE(7, Gq_);

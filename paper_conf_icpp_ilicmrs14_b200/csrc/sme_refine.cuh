@@ -36,6 +36,7 @@ struct SmeParams {
   size_t plane;
   int lambda;                                         // G18 rate term (0 = pure SAD, G13)
   int fence;                                          // outputs are peer memory (me_ipc_open): system fence at exit
+  uint32_t k_hi;                                      // = kAvgHi (vavg4)
 };
 
 // ring-1 spiral order s_k (G12/G14), compile-time so unrolled loops fold it
@@ -162,11 +163,11 @@ __device__ __forceinline__ void half_sad_sweep(const uint8_t* __restrict__ sf, s
 
 // the 8 quarter candidates around half-grid point H from its 3x3 half-grid
 // windows hp[b][a] (rows hy-1..hy+1, columns hx-1..hx+1), O2 averaging rule
-__device__ __forceinline__ uint32_t quarter_win(const uint32_t (&hp)[3][3], int k, bool mixed) {
+__device__ __forceinline__ uint32_t quarter_win(const uint32_t (&hp)[3][3], int k, bool mixed, uint32_t kh) {
   const int dx = k < 2 ? 0 : ((k & 1) ? 1 : -1);
   const int dy = k < 2 ? ((k & 1) ? 1 : -1) : (k < 4 ? -1 : k < 6 ? 0 : 1);
-  if (dx == 0 || dy == 0) return vavg4(hp[1][1], hp[1 + dy][1 + dx]);
-  return vavg4(mixed ? hp[1][1] : hp[1][1 + dx], mixed ? hp[1 + dy][1 + dx] : hp[1 + dy][1]);
+  if (dx == 0 || dy == 0) return vavg4(hp[1][1], hp[1 + dy][1 + dx], kh);
+  return vavg4(mixed ? hp[1][1] : hp[1][1 + dx], mixed ? hp[1 + dy][1 + dx] : hp[1 + dy][1], kh);
 }
 
 // Quarter stage, SAD, one block group of HR rows, around half-grid point (hx, hy):
@@ -176,7 +177,7 @@ __device__ __forceinline__ uint32_t quarter_win(const uint32_t (&hp)[3][3], int 
 // parity) r = 0..HR-1, 4 LDG each, and CF row r uses outer r, middle r, outer r+1.
 template <int HR>
 __device__ __forceinline__ void quarter_sad_sweep(size_t plane, int pitch, const uint8_t* base, int hx, int hy,
-                                                  const uint32_t* cf, uint32_t (&qs)[8]) {
+                                                  const uint32_t* cf, uint32_t (&qs)[8], uint32_t kh) {
   const bool mixed = ((hx ^ hy) & 1) != 0;
   const int xm = hx - 1, x0 = hx, ym = hy - 1, y0 = hy;
   auto at = [&](int X, int Y) {                 // plane row pointer of half-grid point (X, Y), CF row 0
@@ -196,7 +197,7 @@ __device__ __forceinline__ void quarter_sad_sweep(size_t plane, int pitch, const
     if (r > 0) {
       const uint32_t hp[3][3] = {{po[0], po[1], po[2]}, {pm[0], pm[1], pm[2]}, {olr.l, oc, olr.r}};
 #pragma unroll
-      for (int k = 0; k < 8; ++k) qs[k] = vad4(cf[r - 1], quarter_win(hp, k, mixed), qs[k]);
+      for (int k = 0; k < 8; ++k) qs[k] = vad4(cf[r - 1], quarter_win(hp, k, mixed, kh), qs[k]);
     }
     if (r < HR) {
       const Win2 mlr = load_lr(m_lr + r * pitch);
@@ -301,7 +302,7 @@ __device__ __forceinline__ void refine_mode(const SmeParams& P, const uint8_t* _
       const int hx = bvx >> 1, hy = bvy >> 1;          // half-grid coordinates (bvx, bvy even)
       uint32_t qs[8];
       if (!SATD) {                                     // SAD: one row sweep
-        quarter_sad_sweep<4 * YG>(P.plane, P.pitch, sf + (size_t)(yg + P.pad) * P.pitch + (xs + P.pad), hx, hy, cf, qs);
+        quarter_sad_sweep<4 * YG>(P.plane, P.pitch, sf + (size_t)(yg + P.pad) * P.pitch + (xs + P.pad), hx, hy, cf, qs, P.k_hi);
       } else {                                         // SATD: whole 4x4 blocks, one candidate at a time
         const bool mixed = ((hx ^ hy) & 1) != 0;
         int off[3][3];                                 // window offsets from the strip's row base
@@ -333,7 +334,7 @@ __device__ __forceinline__ void refine_mode(const SmeParams& P, const uint8_t* _
               const uint32_t* w0 = reinterpret_cast<const uint32_t*>(e0 & ~uintptr_t(3));
               const uint32_t* w1 = reinterpret_cast<const uint32_t*>(e1 & ~uintptr_t(3));
               smp[r] = vavg4(__funnelshift_r(__ldg(w0), __ldg(w0 + 1), 8u * (uint32_t)(e0 & 3)),
-                             __funnelshift_r(__ldg(w1), __ldg(w1 + 1), 8u * (uint32_t)(e1 & 3)));
+                             __funnelshift_r(__ldg(w1), __ldg(w1 + 1), 8u * (uint32_t)(e1 & 3)), P.k_hi);
             }
             qs[k] += satd4(cf + 4 * jb, smp);
           }
