@@ -52,6 +52,8 @@ def parse():
     ap.add_argument("--me-ctas", type=int, default=None, help="ME_OPT_ME_CTAS_PER_SM")
     ap.add_argument("--fused", type=int, default=None, help="ME_OPT_FUSED_SME")
     ap.add_argument("--adaptive", action="store_true", help="N>1: re-split MB rows every frame (SURVEY §8 f3)")
+    ap.add_argument("--overlap", type=int, default=None,
+                    help="ME_OPT_OVERLAP_SME for the e2e stream (SME(t) co-runs with ME(t+1))")
     ap.add_argument("--exchange", choices=["peer", "collective"], default="peer",
                     help="N>1: stripe+halo pull and SME stores over peer memory (PeerStream) or NCCL "
                          "broadcast + gather (ShardedStream; always used with --adaptive)")
@@ -390,6 +392,8 @@ def run_feves(args, cfg):
     if not args.no_e2e and world == 1:
         qm_h = torch.empty(me.mv_shape() + (2,), dtype=torch.int16).pin_memory()
         qs_h = torch.empty(me.mv_shape(), dtype=torch.uint16).pin_memory()
+        if args.overlap is not None:
+            me.set_option(me.OPT_OVERLAP_SME, args.overlap)
         me.stream_reset()
         for i in range(cfg.n_rf + 2):
             me.stream_push(pinned[i % n_frames], out=(qm_h, qs_h))
@@ -405,7 +409,8 @@ def run_feves(args, cfg):
         e2e = {"value": args.e2e_steps / (e2e_ms / 1e3), "unit": "frames/s",
                "h2d_bytes_per_step": pinned[0].numel(),
                "d2h_bytes_per_step": qm_h.numel() * 2 + qs_h.numel() * 2,
-               "api": "me_stream_push(cf_on_host=1, out_on_host=1), pinned buffers, C-ABI"}
+               "api": "me_stream_push(cf_on_host=1, out_on_host=1), pinned buffers, C-ABI"
+                      + (", ME_OPT_OVERLAP_SME" if args.overlap else "")}
 
     if rank != 0:
         if world > 1:

@@ -71,6 +71,12 @@ struct me_ctx {
   cudaEvent_t ev_me[kMaxRf], ev_sme_done;
   int sf_v0[kMaxRf], sf_v1[kMaxRf];   // MB rows whose SF rows each SF-ring slot holds (re-split support)
   int halo_only;                      // ME_OPT_HALO_ONLY: pushes copy the stripe + halo rows only
+  int overlap;                        // ME_OPT_OVERLAP_SME: SME(t) on its own stream, co-running with ME(t+1)
+  cudaStream_t ov_st;                 // overlap: SME stream (high priority)
+  cudaEvent_t ev_ov_me, ev_ov_sme;    // overlap: ME(t) done, SME(t) done
+  int16_t* d_mvs_ov[2];               // overlap: ME outputs double-buffered (SME(t) reads while ME(t+1) writes)
+  uint16_t* d_sads_ov[2];
+  bool ov_pending;                    // an SME of an earlier push may still run on ov_st
   int fv0[kMaxRf + 2], fv1[kMaxRf + 2];   // frame rows each frame-ring slot holds
   struct Peer { uintptr_t lo, hi; void* base; } peers[16];   // me_ipc_open mappings
   int n_peers;
@@ -234,6 +240,10 @@ extern "C" void me_destroy(me_ctx* c) {
   if (c->own_stream && c->stream) cudaStreamDestroy(c->stream);
   for (int i = 0; i < c->n_peers; ++i)
     if (c->peers[i].base) cudaIpcCloseMemHandle(c->peers[i].base);
+  if (c->ov_st) { cudaStreamSynchronize(c->ov_st); cudaStreamDestroy(c->ov_st); }
+  if (c->ev_ov_me) cudaEventDestroy(c->ev_ov_me);
+  if (c->ev_ov_sme) cudaEventDestroy(c->ev_ov_sme);
+  for (int i = 0; i < 2; ++i) { cudaFree(c->d_mvs_ov[i]); cudaFree(c->d_sads_ov[i]); }
   delete c;
 }
 
@@ -535,6 +545,46 @@ static int stream_alloc(me_ctx* c) {
   return ME_OK;
 }
 
+// ME_OPT_OVERLAP_SME: push t enqueues
+//   side : wait(main fork), wait(SME(t-1) done)   INT(t-1) -> SF slot (t-1) mod n_rf
+//          (that slot held frame t-1-n_rf, which SME(t-1) read as its last RF)
+//   main : ME(t) -> ME buffer t & 1; then wait(SME(t-1) done), so everything later on the
+//          context stream (the next frame copy, ME(t+1), the caller) sees frame t-1 complete
+//   ov_st: wait(ME(t)), wait(INT(t-1))             SME(t) -> outputs
+// so SME(t) (latency-bound) co-runs with ME(t+1) (ALU-bound) of the next push.  The ME
+// outputs are double-buffered because ME(t+1) writes while SME(t) reads.
+static int push_overlapped(me_ctx* c, const uint8_t* cur, const uint8_t* const* rfs, const uint8_t* const* sfs,
+                           const uint8_t* new_rf, uint8_t* new_sf, int16_t* qm, uint16_t* qs, int n_ref, int par) {
+  if (!c->ov_st) {
+    int lo = 0, hi = 0;
+    const size_t nmv = (size_t)c->mb_cols * c->mb_rows * c->n_rf * kNPart;
+    bool ok = cudaDeviceGetStreamPriorityRange(&lo, &hi) == cudaSuccess &&
+              cudaStreamCreateWithPriority(&c->ov_st, cudaStreamNonBlocking, hi) == cudaSuccess &&
+              cudaEventCreateWithFlags(&c->ev_ov_me, cudaEventDisableTiming) == cudaSuccess &&
+              cudaEventCreateWithFlags(&c->ev_ov_sme, cudaEventDisableTiming) == cudaSuccess;
+    for (int i = 0; ok && i < 2; ++i)
+      ok = cudaMalloc(&c->d_mvs_ov[i], nmv * 4) == cudaSuccess && cudaMalloc(&c->d_sads_ov[i], nmv * 2) == cudaSuccess;
+    if (!ok) { cudaGetLastError(); return ME_ENOMEM; }
+  }
+  int st;
+  if (cudaEventRecord(c->ev_fork, c->stream) != cudaSuccess ||
+      cudaStreamWaitEvent(c->side, c->ev_fork, 0) != cudaSuccess ||
+      (c->ov_pending && cudaStreamWaitEvent(c->side, c->ev_ov_sme, 0) != cudaSuccess))
+    return launch_status();
+  if ((st = launch_int(c, new_rf, new_sf, c->side)) != ME_OK) return st;
+  if (cudaEventRecord(c->ev_join, c->side) != cudaSuccess) return launch_status();
+  if ((st = launch_me(c, cur, rfs, c->d_mvs_ov[par], c->d_sads_ov[par], n_ref, c->stream)) != ME_OK) return st;
+  if (cudaEventRecord(c->ev_ov_me, c->stream) != cudaSuccess ||
+      (c->ov_pending && cudaStreamWaitEvent(c->stream, c->ev_ov_sme, 0) != cudaSuccess) ||
+      cudaStreamWaitEvent(c->ov_st, c->ev_ov_me, 0) != cudaSuccess ||
+      cudaStreamWaitEvent(c->ov_st, c->ev_join, 0) != cudaSuccess)
+    return launch_status();
+  if ((st = launch_sme(c, cur, sfs, c->d_mvs_ov[par], c->d_sads_ov[par], qm, qs, n_ref, c->ov_st)) != ME_OK) return st;
+  if (cudaEventRecord(c->ev_ov_sme, c->ov_st) != cudaSuccess) return launch_status();
+  c->ov_pending = true;
+  return ME_OK;
+}
+
 extern "C" int me_stream_push(me_ctx* c, const uint8_t* cf, int cf_on_host, int16_t* out_qmvs,
                               uint16_t* out_qsads, int out_on_host, int* n_ref_used) {
   if (!c || !cf) return ME_EINVAL;
@@ -603,7 +653,9 @@ extern "C" int me_stream_push(me_ctx* c, const uint8_t* cf, int cf_on_host, int1
     uint16_t* qs = (out_qsads && !out_on_host) ? out_qsads : (out_on_host ? c->d_qsads2[par] : c->d_qsads);
     // the device output buffer t & 1 is free once the download of push t-2 finished
     if (out_on_host && cudaStreamWaitEvent(c->stream, c->ev_down[par], 0) != cudaSuccess) return launch_status();
-    if (c->fuse && !c->lambda && !c->satd && !c->inclusive) {
+    if (c->overlap && !c->pipeline && !(c->fuse && !c->lambda && !c->satd && !c->inclusive)) {
+      if ((st = push_overlapped(c, cur, rfs, sfs, new_rf, new_sf, qm, qs, n_ref, par)) != ME_OK) return st;
+    } else if (c->fuse && !c->lambda && !c->satd && !c->inclusive) {
       // fused: the SME of ref 0 reads SF(t-1), so INT(t-1) runs first on the same stream
       if ((st = launch_int(c, new_rf, new_sf, c->stream)) != ME_OK) return st;
       if ((st = launch_me(c, cur, rfs, nullptr, nullptr, n_ref, c->stream, sfs, qm, qs)) != ME_OK) return st;
@@ -617,7 +669,7 @@ extern "C" int me_stream_push(me_ctx* c, const uint8_t* cf, int cf_on_host, int1
       if ((st = run_me_sme(c, cur, rfs, sfs, c->d_mvs, c->d_sads, qm, qs, n_ref, c->ev_join)) != ME_OK) return st;
     }
     const size_t nmv = (size_t)(c->row1 - c->row0) * c->mb_cols * c->n_rf * kNPart;
-    if (cudaEventRecord(c->ev_done[par], c->stream) != cudaSuccess) return launch_status();
+    if (cudaEventRecord(c->ev_done[par], c->ov_pending ? c->ov_st : c->stream) != cudaSuccess) return launch_status();
     if (out_on_host) {   // download on the copy-out stream, overlapping the next frame's compute
       if (cudaStreamWaitEvent(c->copy_out, c->ev_done[par], 0) != cudaSuccess ||
           (out_qmvs && cudaMemcpyAsync(out_qmvs, qm, nmv * 4, cudaMemcpyDeviceToHost, c->copy_out) != cudaSuccess) ||
@@ -639,6 +691,7 @@ extern "C" int me_sync(me_ctx* c) {
   if (e == cudaSuccess && c->copy_out) e = cudaStreamSynchronize(c->copy_out);
   if (e == cudaSuccess && c->side) e = cudaStreamSynchronize(c->side);
   if (e == cudaSuccess && c->sme_st) e = cudaStreamSynchronize(c->sme_st);
+  if (e == cudaSuccess && c->ov_st) e = cudaStreamSynchronize(c->ov_st);
   return e == cudaSuccess ? ME_OK : ME_ECUDA;
 }
 
@@ -690,6 +743,12 @@ extern "C" int me_set_option(me_ctx* c, int option, int value) {
       return ME_OK;
     case ME_OPT_HALO_ONLY:
       c->halo_only = value ? 1 : 0;
+      return ME_OK;
+    case ME_OPT_OVERLAP_SME:
+      if (c->stream) cudaStreamSynchronize(c->stream);
+      if (c->ov_st) cudaStreamSynchronize(c->ov_st);
+      c->ov_pending = false;
+      c->overlap = value ? 1 : 0;
       return ME_OK;
     case ME_OPT_LAMBDA:
       if (value < 0 || value > 2000) return ME_EINVAL;

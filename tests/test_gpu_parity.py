@@ -405,3 +405,40 @@ def test_sa_inclusive(feves, orc, W, H, S, n_rf, kind, lam):
     np.testing.assert_array_equal(m0.cpu().numpy().reshape(n, n_rf, 41, 2), o_m0)
     np.testing.assert_array_equal(s0.cpu().numpy().reshape(n, n_rf, 41), o_s0)
     me.close()
+
+
+@pytest.mark.parametrize("host", [False, True])
+def test_stream_overlap_sme_equals_serial(feves, host):
+    """ME_OPT_OVERLAP_SME (SME(t) co-runs with ME(t+1) on its own stream): every frame's
+    outputs, each pushed into its own buffer, equal the serial stream's, bitwise; with a
+    large frame so that the kernels really overlap, and the RF ramp included."""
+    W, H, S, n_rf = 640, 360, 32, 4
+    frames = [gen_tex(W, H, t, 71) for t in range(9)]
+
+    def run(overlap):
+        me = feves.MotionEstimator(W, H, S, n_rf)
+        me.set_option(me.OPT_OVERLAP_SME, int(overlap))
+        outs = []
+        for f in frames:
+            if host:
+                o = (torch.full(me.mv_shape() + (2,), -7, dtype=torch.int16).pin_memory(),
+                     torch.full(me.mv_shape(), 7, dtype=torch.uint16).pin_memory())
+                src = torch.from_numpy(f).pin_memory()
+            else:
+                o = (torch.full(me.mv_shape() + (2,), -7, dtype=torch.int16, device="cuda"),
+                     torch.full(me.mv_shape(), 7, dtype=torch.uint16, device="cuda"))
+                src = _dev(f)
+            _, _, used = me.stream_push(src, out=o)
+            outs.append((o, used))
+        me.sync()
+        torch.cuda.synchronize()
+        res = [(o[0].cpu().numpy(), o[1].cpu().numpy(), u) for o, u in outs]
+        me.close()
+        return res
+
+    a, b = run(False), run(True)
+    for (qa, sa, ua), (qb, sb, ub) in zip(a, b):
+        assert ua == ub
+        np.testing.assert_array_equal(qa, qb)
+        np.testing.assert_array_equal(sa, sb)
+    assert any(u == n_rf for _, _, u in a)
