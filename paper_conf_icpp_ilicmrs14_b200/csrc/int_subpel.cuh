@@ -178,7 +178,10 @@ __device__ __forceinline__ void int_body(const IntParams& P, int g, int rr) {
 #undef R_
 }
 
-__global__ void __launch_bounds__(128) int_subpel_kernel(const IntParams P) {
+#ifndef FEVES_INT_MINB
+#define FEVES_INT_MINB 1
+#endif
+__global__ void __launch_bounds__(128, FEVES_INT_MINB) int_subpel_kernel(const IntParams P) {
   if (blockIdx.z == gridDim.z - 1) {
     const int g = P.g_lo + blockIdx.x * blockDim.x + threadIdx.x;
     const int rr = P.row_begin + blockIdx.y * blockDim.y + threadIdx.y;

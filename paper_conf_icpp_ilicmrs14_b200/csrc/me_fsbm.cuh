@@ -63,12 +63,18 @@ struct MeParams {
 __host__ __device__ constexpr int me_lx(int S) { return S >= 32 ? 32 : S >= 16 ? 16 : S >= 8 ? 8 : 4; }
 __host__ __device__ constexpr int me_ngx(int S) { return (S + me_lx(S) - 1) / me_lx(S); }
 __host__ __device__ constexpr int me_nsub(int S) { return 32 / me_lx(S); }
-__host__ __device__ constexpr int me_dyl(int S) { return ((S + me_nsub(S) - 1) / me_nsub(S) + kMeT - 1) / kMeT * kMeT; }
+// warps splitting the dy range: at S = 16 (CIF, 396 MBs, one RF) a second warp takes the
+// other half of the dy range, doubling the warps of a grid too small to fill the GPU
+// (ME 10.9 -> 9.0 us).  Measured slower for S = 32 (69.9 -> 73.4 us), so only S = 16.
+__host__ __device__ constexpr int me_nwy(int S) { return S == 16 ? 2 : 1; }
+__host__ __device__ constexpr int me_dyl(int S) {
+  return ((S + me_nsub(S) * me_nwy(S) - 1) / (me_nsub(S) * me_nwy(S)) + kMeT - 1) / kMeT * kMeT;
+}
 __host__ __device__ constexpr int me_pw(int S) { return (((S - 1) >> 2) + 4 + 3) & ~3; }   // words/row, %4 == 0
 __host__ __device__ constexpr int me_cstride(int S) {                                      // == 8 (mod 32)
   return (S + 15) * me_pw(S) + ((8 - ((S + 15) * me_pw(S)) % 32) % 32 + 32) % 32;
 }
-__host__ __device__ constexpr int me_threads(int S) { return 32 * me_ngx(S); }
+__host__ __device__ constexpr int me_threads(int S) { return 32 * me_ngx(S) * me_nwy(S); }
 __host__ __device__ constexpr int me_smem_words(int S) { return 64 + 4 * me_cstride(S) + (me_threads(S) / 32) * kNPart; }
 // + fused SME: the ME winners of every RF (packed MV, SAD) stay in shared memory
 __host__ __device__ constexpr int me_smem_words_fused(int S, int n_rf) { return me_smem_words(S) + 2 * n_rf * kNPart; }
@@ -305,8 +311,8 @@ __global__ void __launch_bounds__(S_CT ? 128 : 256, S_CT ? FEVES_ME_MINB : 2) me
   const int nwarps = blockDim.x >> 5;
 
   // ---- lane geometry: dx column and dy sub-range ----
-  const int gx = warp % NGX;
-  const int xi = lane % LX, sub = lane / LX;
+  const int gx = warp % NGX, wy = me_nwy(S) > 1 ? warp / NGX : 0;
+  const int xi = lane % LX, sub = wy * NSUB + lane / LX;
   const int dx = min(-R + gx * LX + xi, hi);               // beyond-range lanes duplicate dx=hi
   const int off = dx + R;                                  // byte offset inside the window row
   const uint32_t* wbase = win + (off & 3) * CSTRIDE + (off >> 2);
