@@ -108,17 +108,21 @@ __device__ __forceinline__ uint32_t strip_block_dist(const uint8_t* __restrict__
 // (left) and a+1 (right) are both funnel shifts of them (the right one with the
 // clamped shift, 32 -> the high word).  One pair of LDG per row serves the two
 // horizontally adjacent half-grid windows of the SME (same plane, columns x, x+1).
+// The SF pitch and plane size are multiples of 16 bytes (G11 layout), so a
+// sweep's rows share one alignment: the aligned word pointer and the byte shift
+// are computed once per sweep (RowP) and each row costs 2 LDG + the funnel shifts.
 struct Win2 { uint32_t l, r; };
-__device__ __forceinline__ Win2 load_lr(const uint8_t* __restrict__ p) {
+struct RowP { const uint32_t* w; uint32_t sh; };
+__device__ __forceinline__ RowP rowp(const uint8_t* p) {
   const uintptr_t a = reinterpret_cast<uintptr_t>(p);
-  const uint32_t* w = reinterpret_cast<const uint32_t*>(a & ~uintptr_t(3));
-  const uint32_t w0 = __ldg(w), w1 = __ldg(w + 1), sh = 8u * (uint32_t)(a & 3);
-  return {__funnelshift_r(w0, w1, sh), __funnelshift_rc(w0, w1, sh + 8u)};
+  return {reinterpret_cast<const uint32_t*>(a & ~uintptr_t(3)), 8u * (uint32_t)(a & 3)};
 }
-__device__ __forceinline__ uint32_t load_w(const uint8_t* __restrict__ p) {
-  const uintptr_t a = reinterpret_cast<uintptr_t>(p);
-  const uint32_t* w = reinterpret_cast<const uint32_t*>(a & ~uintptr_t(3));
-  return __funnelshift_r(__ldg(w), __ldg(w + 1), 8u * (uint32_t)(a & 3));
+__device__ __forceinline__ Win2 ld_lr(const RowP& q, int off) {   // off = row * (pitch / 4)
+  const uint32_t w0 = __ldg(q.w + off), w1 = __ldg(q.w + off + 1);
+  return {__funnelshift_r(w0, w1, q.sh), __funnelshift_rc(w0, w1, q.sh + 8u)};
+}
+__device__ __forceinline__ uint32_t ld_w(const RowP& q, int off) {
+  return __funnelshift_r(__ldg(q.w + off), __ldg(q.w + off + 1), q.sh);
 }
 
 // Half stage, SAD, one block group of HR rows (DESIGN.md §6 "row sweep"): for the
@@ -136,17 +140,18 @@ __device__ __forceinline__ void half_sad_sweep(const uint8_t* __restrict__ sf, s
                                                const uint8_t* base, int mx, int my, const uint32_t* cf,
                                                uint32_t (&sad)[8]) {
   // base = plane 0 at the strip's top-left integer sample (pad applied)
-  const uint8_t* ph = base + 8 * plane + (ptrdiff_t)(my - 1) * pitch + mx;
-  const uint8_t* pj = base + 10 * plane + (ptrdiff_t)(my - 1) * pitch + (mx - 1);
-  const uint8_t* pb = base + 2 * plane + (ptrdiff_t)my * pitch + (mx - 1);
+  const RowP ph = rowp(base + 8 * plane + (ptrdiff_t)(my - 1) * pitch + mx);
+  const RowP pj = rowp(base + 10 * plane + (ptrdiff_t)(my - 1) * pitch + (mx - 1));
+  const RowP pb = rowp(base + 2 * plane + (ptrdiff_t)my * pitch + (mx - 1));
+  const int wp = pitch >> 2;
 #pragma unroll
   for (int k = 0; k < 8; ++k) sad[k] = 0;
 #pragma unroll
   for (int r = 0; r <= HR; ++r) {
-    const uint32_t hw = load_w(ph + r * pitch);
-    const Win2 jw = load_lr(pj + r * pitch);
+    const uint32_t hw = ld_w(ph, r * wp);
+    const Win2 jw = ld_lr(pj, r * wp);
     if (r < HR) {
-      const Win2 bw = load_lr(pb + r * pitch);
+      const Win2 bw = ld_lr(pb, r * wp);
       sad[0] = vad4(cf[r], hw, sad[0]);
       sad[2] = vad4(cf[r], jw.l, sad[2]);
       sad[3] = vad4(cf[r], jw.r, sad[3]);
@@ -183,25 +188,26 @@ __device__ __forceinline__ void quarter_sad_sweep(size_t plane, int pitch, const
   auto at = [&](int X, int Y) {                 // plane row pointer of half-grid point (X, Y), CF row 0
     return base + (size_t)(8 * (Y & 1) + 2 * (X & 1)) * plane + (ptrdiff_t)(Y >> 1) * pitch + (X >> 1);
   };
-  const uint8_t* o_lr = at(xm, ym);             // outer rows, columns hx-1 / hx+1
-  const uint8_t* o_c = at(x0, ym);              // outer rows, column hx
-  const uint8_t* m_lr = at(xm, y0);             // middle rows
-  const uint8_t* m_c = at(x0, y0);
+  const RowP o_lr = rowp(at(xm, ym));           // outer rows, columns hx-1 / hx+1
+  const RowP o_c = rowp(at(x0, ym));            // outer rows, column hx
+  const RowP m_lr = rowp(at(xm, y0));           // middle rows
+  const RowP m_c = rowp(at(x0, y0));
+  const int wp = pitch >> 2;
 #pragma unroll
   for (int k = 0; k < 8; ++k) qs[k] = 0;
   uint32_t po[3], pm[3];                        // previous outer / middle windows (L, C, R)
 #pragma unroll
   for (int r = 0; r <= HR; ++r) {
-    const Win2 olr = load_lr(o_lr + r * pitch);
-    const uint32_t oc = load_w(o_c + r * pitch);
+    const Win2 olr = ld_lr(o_lr, r * wp);
+    const uint32_t oc = ld_w(o_c, r * wp);
     if (r > 0) {
       const uint32_t hp[3][3] = {{po[0], po[1], po[2]}, {pm[0], pm[1], pm[2]}, {olr.l, oc, olr.r}};
 #pragma unroll
       for (int k = 0; k < 8; ++k) qs[k] = vad4(cf[r - 1], quarter_win(hp, k, mixed, kh), qs[k]);
     }
     if (r < HR) {
-      const Win2 mlr = load_lr(m_lr + r * pitch);
-      pm[0] = mlr.l; pm[1] = load_w(m_c + r * pitch); pm[2] = mlr.r;
+      const Win2 mlr = ld_lr(m_lr, r * wp);
+      pm[0] = mlr.l; pm[1] = ld_w(m_c, r * wp); pm[2] = mlr.r;
       po[0] = olr.l; po[1] = oc; po[2] = olr.r;
     }
   }
