@@ -260,8 +260,14 @@ __device__ __forceinline__ void refine_mode(const SmeParams& P, const uint8_t* _
   for (int g = 0; g < NG; ++g) {
     const int yg = ys0 + 4 * g * YG;   // first frame row of this group
     uint32_t cf[4 * YG];               // this group's CF strip rows
+    if ((P.W & 3) == 0 && xs + 3 < P.W && yg + 4 * YG <= P.H) {   // inside the frame: aligned words
+      const uint32_t* c0 = reinterpret_cast<const uint32_t*>(P.cf + (size_t)yg * P.W + xs);
 #pragma unroll
-    for (int r = 0; r < 4 * YG; ++r) cf[r] = load4_clamped(P.cf, P.W, P.H, xs, yg + r);
+      for (int r = 0; r < 4 * YG; ++r) cf[r] = __ldg(c0 + r * (P.W >> 2));
+    } else {                                                      // clamped (G5, G6)
+#pragma unroll
+      for (int r = 0; r < 4 * YG; ++r) cf[r] = load4_clamped(P.cf, P.W, P.H, xs, yg + r);
+    }
     const int p = mode_part<MODE>(bx, g * YG);
     const uint32_t mv = __ldg(P.in_mvs + o + p);
     int bvx = 4 * (int)(int16_t)(mv & 0xffffu);
