@@ -11,6 +11,7 @@
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
+#include <algorithm>
 #include <mutex>
 #include <vector>
 
@@ -141,13 +142,21 @@ static int upload_key_table(me_ctx* c) {
   c->kshift = c->lambda ? 15 : 16;
   c->kmul = 1u << c->kshift;
   std::vector<uint32_t> e((size_t)Sc * Sc), inv((size_t)(c->S + 1) * (c->S + 1), 0);
+  // DENSE rank: the candidates of the SA numbered 0..Sc^2-1 in spiral order (G4).  It
+  // orders candidates exactly as the spiral rank does, and < 4096 for S <= 64 is what
+  // lets the ME kernel build parent keys as sums of child keys (me_fsbm.cuh, kSumKeys).
+  std::vector<std::pair<int, uint32_t>> order;
+  order.reserve((size_t)Sc * Sc);
   for (int dy = -c->R; dy <= hi; ++dy)
-    for (int dx = -c->R; dx <= hi; ++dx) {
-      const int r = spiral_rank_closed_form(dx, dy);
-      e[(size_t)(dy + c->R) * Sc + (dx + c->R)] =
-          (uint32_t)(c->lambda * (se_bits(4 * dx) + se_bits(4 * dy))) * c->kmul + (uint32_t)r;
-      inv[r] = (uint32_t)(uint16_t)dx | ((uint32_t)(uint16_t)dy << 16);
-    }
+    for (int dx = -c->R; dx <= hi; ++dx)
+      order.emplace_back(spiral_rank_closed_form(dx, dy), (uint32_t)(uint16_t)dx | ((uint32_t)(uint16_t)dy << 16));
+  std::sort(order.begin(), order.end());
+  for (size_t r = 0; r < order.size(); ++r) {
+    const int dx = (int)(int16_t)(order[r].second & 0xffffu), dy = (int)(int16_t)(order[r].second >> 16);
+    e[(size_t)(dy + c->R) * Sc + (dx + c->R)] =
+        (uint32_t)(c->lambda * (se_bits(4 * dx) + se_bits(4 * dy))) * c->kmul + (uint32_t)r;
+    inv[r] = order[r].second;
+  }
   c->me_threads = me_threads(Sc);
   c->me_smem = (size_t)me_smem_words(Sc) * 4;
   c->me_smem_fused = (size_t)me_smem_words_fused(Sc, c->n_rf) * 4;
