@@ -29,7 +29,7 @@ struct me_ctx {
   int device;
   cudaStream_t stream;
   bool own_stream;
-  uint32_t* d_rank;      // [S][S]
+  uint32_t* d_rank;      // [S][Sp]: [dx+R][dy+R], column pitch Sp = S rounded up to 4 (me_rank_pitch)
   uint32_t* d_inv;       // [(S+1)^2]
   int16_t* d_mvs;        // scratch for me_encode_frame (full frame)
   uint16_t* d_sads;
@@ -141,10 +141,11 @@ static int upload_key_table(me_ctx* c) {
   const int Sc = c->S + c->inclusive, hi = Sc - 1 - c->R;   // candidates per axis, dx,dy in [-R, hi]
   c->kshift = c->lambda ? 15 : 16;
   c->kmul = 1u << c->kshift;
-  std::vector<uint32_t> e((size_t)Sc * Sc), inv((size_t)(c->S + 1) * (c->S + 1), 0);
+  const int Sp = me_rank_pitch(Sc);
+  std::vector<uint32_t> e((size_t)Sc * Sp, 0), inv((size_t)(c->S + 1) * (c->S + 1), 0);
   // DENSE rank: the candidates of the SA numbered 0..Sc^2-1 in spiral order (G4).  It
   // orders candidates exactly as the spiral rank does, and < 4096 for S <= 64 is what
-  // lets the ME kernel build parent keys as sums of child keys (me_fsbm.cuh, kSumKeys).
+  // lets the ME kernel build parent keys as sums of child keys (me_fsbm.cuh, SumKeys).
   std::vector<std::pair<int, uint32_t>> order;
   order.reserve((size_t)Sc * Sc);
   for (int dy = -c->R; dy <= hi; ++dy)
@@ -153,7 +154,7 @@ static int upload_key_table(me_ctx* c) {
   std::sort(order.begin(), order.end());
   for (size_t r = 0; r < order.size(); ++r) {
     const int dx = (int)(int16_t)(order[r].second & 0xffffu), dy = (int)(int16_t)(order[r].second >> 16);
-    e[(size_t)(dy + c->R) * Sc + (dx + c->R)] =
+    e[(size_t)(dx + c->R) * Sp + (dy + c->R)] =
         (uint32_t)(c->lambda * (se_bits(4 * dx) + se_bits(4 * dy))) * c->kmul + (uint32_t)r;
     inv[r] = order[r].second;
   }
@@ -193,7 +194,7 @@ extern "C" me_ctx* me_create(int width, int height, int sa_range, int n_rf) {
   c->me_ctas_per_sm = 0;
 
   const size_t nmv = (size_t)c->mb_cols * c->mb_rows * n_rf * kNPart;
-  bool ok = cudaMalloc(&c->d_rank, (size_t)(S + 1) * (S + 1) * 4) == cudaSuccess &&
+  bool ok = cudaMalloc(&c->d_rank, (size_t)(S + 1) * me_rank_pitch(S + 1) * 4) == cudaSuccess &&
             cudaMalloc(&c->d_inv, (size_t)(S + 1) * (S + 1) * 4) == cudaSuccess &&
             cudaMalloc(&c->d_mvs, nmv * 4) == cudaSuccess &&
             cudaMalloc(&c->d_sads, nmv * 2) == cudaSuccess &&

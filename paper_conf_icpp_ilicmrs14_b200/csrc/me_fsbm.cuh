@@ -43,7 +43,7 @@ struct MeParams {
   int W, H, S, R, n_rf;       // S = candidates per axis (sa_range, +1 if inclusive); n_rf = RFs searched
   int rf_stride;              // RF dimension of the output layout (the context's n_rf)
   int mb_cols, row0;
-  const uint32_t* rank_tab;   // [S][S] (S candidates per axis), [dy+R][dx+R] -> key addend E =
+  const uint32_t* rank_tab;   // [S][Sp] (S candidates per axis), [dx+R][dy+R] -> key addend E =
                               // lambda*R(4dx,4dy)*kmul + spiral rank (G4, G18)
   const uint32_t* inv_tab;    // rank -> (dx & 0xffff) | (dy << 16)
   uint32_t kmul;              // key = J * kmul + rank: 2^16 (lambda = 0) or 2^15 (J may exceed 16 bits)
@@ -74,6 +74,8 @@ __host__ __device__ constexpr int me_pw(int S) { return (((S - 1) >> 2) + 4 + 3)
 __host__ __device__ constexpr int me_cstride(int S) {                                      // == 8 (mod 32)
   return (S + 15) * me_pw(S) + ((8 - ((S + 15) * me_pw(S)) % 32) % 32 + 32) % 32;
 }
+// rank table column pitch: a lane's T = 4 consecutive dy are one aligned 16-byte load
+__host__ __device__ constexpr int me_rank_pitch(int S) { return (S + 3) & ~3; }
 __host__ __device__ constexpr int me_threads(int S) { return 32 * me_ngx(S) * me_nwy(S); }
 __host__ __device__ constexpr int me_smem_words(int S) { return 64 + 4 * me_cstride(S) + (me_threads(S) / 32) * kNPart; }
 // + fused SME: the ME winners of every RF (packed MV, SAD) stay in shared memory
@@ -413,22 +415,27 @@ __global__ void __launch_bounds__(S_CT ? 128 : 256, S_CT ? FEVES_ME_MINB : 2) me
 #pragma unroll
     for (int p = 0; p < kNPart; ++p) M[p] = 0xffffffffu;
 
-    const uint32_t* rank_col = P.rank_tab + off;
+    // the lane's rank column (dy contiguous): with a compile-time S (a multiple of 4)
+    // every chunk start dy0 + R is a multiple of 4, so a chunk's ranks are ONE LDG.128
+    const uint32_t* rank_col = P.rank_tab + off * me_rank_pitch(S) + R;
     uint32_t rank_next[kMeT];
-    {
-      const int dy0 = min(dy_begin, hi + 1 - kMeT);
+    auto load_ranks = [&](int d0) {
+      if (S_CT > 0 && kMeT == 4) {
+        const uint4 v = __ldg(reinterpret_cast<const uint4*>(rank_col + d0));
+        rank_next[0] = v.x; rank_next[1] = v.y; rank_next[2] = v.z; rank_next[3] = v.w;
+      } else {
 #pragma unroll
-      for (int t = 0; t < kMeT; ++t) rank_next[t] = __ldg(rank_col + (dy0 + t + R) * S);
-    }
+        for (int t = 0; t < kMeT; ++t) rank_next[t] = __ldg(rank_col + d0 + t);
+      }
+    };
+    load_ranks(min(dy_begin, hi + 1 - kMeT));
     for (int c = 0; c < DYL; c += kMeT) {
       const int dy0 = min(dy_begin + c, hi + 1 - kMeT);   // clamped chunk: duplicates are harmless
       uint32_t rank[kMeT];
 #pragma unroll
       for (int t = 0; t < kMeT; ++t) rank[t] = rank_next[t];
       {                                                   // prefetch the next chunk's ranks
-        const int dn = min(dy_begin + c + kMeT, hi + 1 - kMeT);
-#pragma unroll
-        for (int t = 0; t < kMeT; ++t) rank_next[t] = __ldg(rank_col + (dn + t + R) * S);
+        load_ranks(min(dy_begin + c + kMeT, hi + 1 - kMeT));
       }
       const uint32_t* wrow = wbase + (dy0 + R) * PW;
 
