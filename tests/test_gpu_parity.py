@@ -53,6 +53,8 @@ SMALL = [  # (W, H, S, n_rf, kind)
     (72, 52, 32, 2, "tex"),            # ragged: 72 = 4.5 MBs, 52 = 3.25 MBs
     (100, 36, 4, 3, "noise"), (50, 30, 6, 1, "tex"), (96, 80, 64, 1, "tex"),
     (48, 48, 12, 2, "flat"), (40, 40, 128, 1, "noise"),
+    # runtime-S kernel where the last staged word of a window row is read (PW == (S-1)/4 + 4)
+    (70, 50, 18, 1, "noise"), (96, 70, 66, 1, "noise"),
 ]
 
 
