@@ -256,8 +256,18 @@ __device__ __forceinline__ void refine_mode(const SmeParams& P, const uint8_t* _
   constexpr int NG = 4 / YG;           // partitions (block groups) inside this lane's strip
   // The groups are refined one after the other (latency-bound kernel: fewer live
   // registers -> more resident warps beats the ILP of refining all NG at once).
+  // the next group's ME result (MV, SAD) is loaded one group ahead, so only the first
+  // group pays the dependent MV -> SF-address round trip
+  uint32_t mv_n = __ldg(P.in_mvs + o + mode_part<MODE>(bx, 0));
+  uint32_t sad_n = (P.in_sads && !SATD) ? (uint32_t)__ldg(P.in_sads + o + mode_part<MODE>(bx, 0)) : 0u;
 #pragma unroll 1
   for (int g = 0; g < NG; ++g) {
+    const uint32_t mv = mv_n, sad_me = sad_n;
+    if (g + 1 < NG) {
+      const int pn = mode_part<MODE>(bx, (g + 1) * YG);
+      mv_n = __ldg(P.in_mvs + o + pn);
+      if (P.in_sads && !SATD) sad_n = __ldg(P.in_sads + o + pn);
+    }
     const int yg = ys0 + 4 * g * YG;   // first frame row of this group
     uint32_t cf[4 * YG];               // this group's CF strip rows
     if ((P.W & 3) == 0 && xs + 3 < P.W && yg + 4 * YG <= P.H) {   // inside the frame: aligned words
@@ -269,12 +279,11 @@ __device__ __forceinline__ void refine_mode(const SmeParams& P, const uint8_t* _
       for (int r = 0; r < 4 * YG; ++r) cf[r] = load4_clamped(P.cf, P.W, P.H, xs, yg + r);
     }
     const int p = mode_part<MODE>(bx, g * YG);
-    const uint32_t mv = __ldg(P.in_mvs + o + p);
     int bvx = 4 * (int)(int16_t)(mv & 0xffffu);
     int bvy = 4 * (int)(int16_t)(mv >> 16);
     uint32_t best;
     if (P.in_sads && !SATD) {
-      best = __ldg(P.in_sads + o + p);
+      best = sad_me;
     } else {
       uint32_t s = 0;
 #pragma unroll
