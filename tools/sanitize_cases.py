@@ -6,7 +6,7 @@ import torch
 import paper_conf_icpp_ilicmrs14_b200 as F
 from synth import gen_tex
 
-for (W, H, S, n) in [(64, 48, 16, 2), (37, 29, 8, 1), (96, 80, 64, 2), (48, 40, 128, 1)]:
+for (W, H, S, n) in [(64, 48, 16, 2), (37, 29, 8, 1), (96, 80, 64, 2), (48, 40, 128, 1), (160, 96, 32, 2), (70, 50, 18, 1)]:
     frames = [torch.from_numpy(gen_tex(W, H, t, 1)).cuda() for t in range(n + 2)]
     me = F.MotionEstimator(W, H, S, n)
     sfs = [me.new_sf() for _ in range(n)]
