@@ -31,6 +31,7 @@ struct me_ctx {
   bool own_stream;
   uint32_t* d_rank;      // [S][Sp]: [dx+R][dy+R], column pitch Sp = S rounded up to 4 (me_rank_pitch)
   uint32_t* d_inv;       // [(S+1)^2]
+  uint32_t* d_glob;      // [4][4096]: S = 128 quadrant-local rank -> global dense rank
   int16_t* d_mvs;        // scratch for me_encode_frame (full frame)
   uint16_t* d_sads;
   // ME launch geometry
@@ -152,17 +153,29 @@ static int upload_key_table(me_ctx* c) {
     for (int dx = -c->R; dx <= hi; ++dx)
       order.emplace_back(spiral_rank_closed_form(dx, dy), (uint32_t)(uint16_t)dx | ((uint32_t)(uint16_t)dy << 16));
   std::sort(order.begin(), order.end());
+  // S = 128, pure SAD: the ME kernel sums keys quadrant by quadrant (me_fsbm.cuh QuadKeys),
+  // so its table holds the rank inside the candidate's quadrant, and glob maps it back
+  const bool quad = c->S == 128 && !c->inclusive && !c->lambda;
+  std::vector<uint32_t> glob(4 * 4096, 0);
+  int qn[4] = {0, 0, 0, 0};
   for (size_t r = 0; r < order.size(); ++r) {
     const int dx = (int)(int16_t)(order[r].second & 0xffffu), dy = (int)(int16_t)(order[r].second >> 16);
+    uint32_t key_rank = (uint32_t)r;
+    if (quad) {
+      const int q = 2 * (dy >= 0) + (dx >= 0);
+      glob[q * 4096 + qn[q]] = (uint32_t)r;
+      key_rank = (uint32_t)qn[q]++;
+    }
     e[(size_t)(dx + c->R) * Sp + (dy + c->R)] =
-        (uint32_t)(c->lambda * (se_bits(4 * dx) + se_bits(4 * dy))) * c->kmul + (uint32_t)r;
+        (uint32_t)(c->lambda * (se_bits(4 * dx) + se_bits(4 * dy))) * c->kmul + key_rank;
     inv[r] = order[r].second;
   }
   c->me_threads = me_threads(Sc);
   c->me_smem = (size_t)me_smem_words(Sc) * 4;
   c->me_smem_fused = (size_t)me_smem_words_fused(Sc, c->n_rf) * 4;
   return cudaMemcpy(c->d_rank, e.data(), e.size() * 4, cudaMemcpyHostToDevice) == cudaSuccess &&
-                 cudaMemcpy(c->d_inv, inv.data(), inv.size() * 4, cudaMemcpyHostToDevice) == cudaSuccess
+                 cudaMemcpy(c->d_inv, inv.data(), inv.size() * 4, cudaMemcpyHostToDevice) == cudaSuccess &&
+                 cudaMemcpy(c->d_glob, glob.data(), glob.size() * 4, cudaMemcpyHostToDevice) == cudaSuccess
              ? ME_OK
              : ME_ECUDA;
 }
@@ -196,6 +209,7 @@ extern "C" me_ctx* me_create(int width, int height, int sa_range, int n_rf) {
   const size_t nmv = (size_t)c->mb_cols * c->mb_rows * n_rf * kNPart;
   bool ok = cudaMalloc(&c->d_rank, (size_t)(S + 1) * me_rank_pitch(S + 1) * 4) == cudaSuccess &&
             cudaMalloc(&c->d_inv, (size_t)(S + 1) * (S + 1) * 4) == cudaSuccess &&
+            cudaMalloc(&c->d_glob, (size_t)4 * 4096 * 4) == cudaSuccess &&
             cudaMalloc(&c->d_mvs, nmv * 4) == cudaSuccess &&
             cudaMalloc(&c->d_sads, nmv * 2) == cudaSuccess &&
             cudaStreamCreateWithFlags(&c->stream, cudaStreamNonBlocking) == cudaSuccess;
@@ -223,6 +237,7 @@ extern "C" void me_destroy(me_ctx* c) {
   if (c->sme_st) cudaStreamSynchronize(c->sme_st);
   cudaFree(c->d_rank);
   cudaFree(c->d_inv);
+  cudaFree(c->d_glob);
   cudaFree(c->d_mvs);
   cudaFree(c->d_sads);
   cudaFree(c->ring);
@@ -312,7 +327,7 @@ static int launch_me(me_ctx* c, const uint8_t* cf, const uint8_t* const* rfs, in
   for (int k = 0; k < n_ref; ++k) P.rf[k] = rfs[k];
   P.W = c->W; P.H = c->H; P.S = c->S + c->inclusive; P.R = c->R; P.n_rf = n_ref; P.rf_stride = c->n_rf;
   P.mb_cols = c->mb_cols; P.row0 = c->row0;
-  P.rank_tab = c->d_rank; P.inv_tab = c->d_inv;
+  P.rank_tab = c->d_rank; P.inv_tab = c->d_inv; P.glob_tab = c->d_glob;
   P.kmul = c->kmul; P.kshift = c->kshift; P.lambda = c->lambda;
   P.out_mvs = mvs; P.out_sads = sads;
   bool vec = (c->W % 16 == 0) && (c->R % 16 == 0);

@@ -46,6 +46,7 @@ struct MeParams {
   const uint32_t* rank_tab;   // [S][Sp] (S candidates per axis), [dx+R][dy+R] -> key addend E =
                               // lambda*R(4dx,4dy)*kmul + spiral rank (G4, G18)
   const uint32_t* inv_tab;    // rank -> (dx & 0xffff) | (dy << 16)
+  const uint32_t* glob_tab;   // S = 128 quadrant key-sum: [quadrant][local rank] -> global dense rank
   uint32_t kmul;              // key = J * kmul + rank: 2^16 (lambda = 0) or 2^15 (J may exceed 16 bits)
   int kshift, lambda;
   int16_t* out_mvs;
@@ -71,13 +72,22 @@ __host__ __device__ constexpr int me_dyl(int S) {
   return ((S + me_nsub(S) * me_nwy(S) - 1) / (me_nsub(S) * me_nwy(S)) + kMeT - 1) / kMeT * kMeT;
 }
 __host__ __device__ constexpr int me_pw(int S) { return (((S - 1) >> 2) + 4 + 3) & ~3; }   // words/row, %4 == 0
+// window rows staged at once: the whole (S+15)-row window, or at S = 128 one dy half of it
+// (S/2 + 15 rows; the window then costs 46 KB instead of 82 KB of shared memory per CTA,
+// so 4 CTAs = 16 warps fit per SM instead of 2 CTAs = 8 warps)
+__host__ __device__ constexpr int me_nstage(int S) { return S == 128 ? 2 : 1; }
+__host__ __device__ constexpr int me_win_rows(int S) { return S / me_nstage(S) + 15; }
 __host__ __device__ constexpr int me_cstride(int S) {                                      // == 8 (mod 32)
-  return (S + 15) * me_pw(S) + ((8 - ((S + 15) * me_pw(S)) % 32) % 32 + 32) % 32;
+  return me_win_rows(S) * me_pw(S) + ((8 - (me_win_rows(S) * me_pw(S)) % 32) % 32 + 32) % 32;
 }
 // rank table column pitch: a lane's T = 4 consecutive dy are one aligned 16-byte load
 __host__ __device__ constexpr int me_rank_pitch(int S) { return (S + 3) & ~3; }
 __host__ __device__ constexpr int me_threads(int S) { return 32 * me_ngx(S) * me_nwy(S); }
-__host__ __device__ constexpr int me_smem_words(int S) { return 64 + 4 * me_cstride(S) + (me_threads(S) / 32) * kNPart; }
+// reduction buffer: [nwarps][halves][41]; two dy halves at S = 128 (QuadKeys)
+__host__ __device__ constexpr int me_red_halves(int S) { return S == 128 ? 2 : 1; }
+__host__ __device__ constexpr int me_smem_words(int S) {
+  return 64 + 4 * me_cstride(S) + (me_threads(S) / 32) * me_red_halves(S) * kNPart;
+}
 // + fused SME: the ME winners of every RF (packed MV, SAD) stay in shared memory
 __host__ __device__ constexpr int me_smem_words_fused(int S, int n_rf) { return me_smem_words(S) + 2 * n_rf * kNPart; }
 
@@ -166,8 +176,16 @@ __device__ __forceinline__ void block_row_keys(const uint32_t (&L)[4], uint32_t 
 // still (SAD, rank).  Every parent key is then ONE IMAD (key_a * 1 + key_b, FMA
 // pipe, opaque 1) and no plain SAD sum is needed: 41 FMA-pipe ops per candidate
 // instead of 54.  The rank is recovered as (key & 0xffff) >> log2(n).
+// S = 128 (16384 candidates) runs the same scheme QUADRANT by quadrant: the rank table
+// then holds each candidate's dense rank INSIDE its quadrant (dx < 0 / >= 0, dy < 0 / >= 0;
+// 4096 each, in spiral order), a warp's dx all lie in one quadrant column, and the dy sweep
+// is cut at dy = 0; after each half the warp minima are stored and the CTA epilogue maps
+// (quadrant, local rank) -> global dense rank (glob_tab) and compares SAD * 2^14 + global
+// rank (SAD < 2^16, rank < 2^14: 30 bits) -- the same (SAD, spiral rank) order (G4).
 template <int S_CT, int KSH>
-struct SumKeys { static constexpr bool value = S_CT > 0 && S_CT <= 64 && KSH == 16; };
+struct SumKeys { static constexpr bool value = S_CT > 0 && S_CT <= 128 && KSH == 16; };
+template <int S_CT, int KSH>
+struct QuadKeys { static constexpr bool value = SumKeys<S_CT, KSH>::value && S_CT == 128; };
 
 __host__ __device__ constexpr int part_log2n(int p) {   // log2(number of 4x4 blocks of partition p, G7)
   return p == 0 ? 4 : p < 5 ? 3 : p < 9 ? 2 : p < 25 ? 1 : 0;
@@ -350,8 +368,10 @@ __global__ void __launch_bounds__(S_CT ? 128 : 256, S_CT ? FEVES_ME_MINB : 2) me
   const int NSUB = me_nsub(S), DYL = me_dyl(S);
   uint32_t* cf_s = smem;                                  // 16 rows x 4 words
   uint32_t* win = smem + 64;                              // 4 copies x CSTRIDE words
-  uint32_t* red = win + 4 * CSTRIDE;                      // [nwarps][41]
-  uint32_t* win_mv = red + (blockDim.x >> 5) * kNPart;    // FUSE: [n_rf][41] packed MVs, then SADs
+  constexpr bool QUAD = QuadKeys<S_CT, KSH>::value;
+  constexpr int NH = QUAD ? 2 : 1;                        // dy halves reduced separately
+  uint32_t* red = win + 4 * CSTRIDE;                      // [nwarps][NH][41]
+  uint32_t* win_mv = red + (blockDim.x >> 5) * me_red_halves(S) * kNPart;   // FUSE: [n_rf][41] MVs, then SADs
   uint32_t* win_sad = win_mv + P.n_rf * kNPart;
 
   const int mbx = blockIdx.x, mby = P.row0 + blockIdx.y;
@@ -372,10 +392,33 @@ __global__ void __launch_bounds__(S_CT ? 128 : 256, S_CT ? FEVES_ME_MINB : 2) me
     cf_s[i] = load4_clamped(P.cf, P.W, P.H, 16 * mbx + 4 * (i & 3), 16 * mby + (i >> 2));
 
   const int xw0 = 16 * mbx - R, yw0 = 16 * mby - R;
-  const int win_rows = S + 15;
+  constexpr int NSTG = S_CT ? me_nstage(S_CT) : 1;      // window stagings per RF (dy halves)
+  const int win_rows = S_CT ? me_win_rows(S_CT) : S + 15;
 
   for (int ref = 0; ref < P.n_rf; ++ref) {
     const uint8_t* __restrict__ rf = P.rf[ref];
+    uint32_t M[kNPart];
+#pragma unroll
+    for (int p = 0; p < kNPart; ++p) M[p] = 0xffffffffu;
+
+    // the lane's rank column (dy contiguous): with a compile-time S (a multiple of 4)
+    // every chunk start dy0 + R is a multiple of 4, so a chunk's ranks are ONE LDG.128
+    const uint32_t* rank_col = P.rank_tab + off * me_rank_pitch(S) + R;
+    uint32_t rank_next[kMeT];
+    auto load_ranks = [&](int d0) {
+      if (S_CT > 0 && kMeT == 4) {
+        const uint4 v = __ldg(reinterpret_cast<const uint4*>(rank_col + d0));
+        rank_next[0] = v.x; rank_next[1] = v.y; rank_next[2] = v.z; rank_next[3] = v.w;
+      } else {
+#pragma unroll
+        for (int t = 0; t < kMeT; ++t) rank_next[t] = __ldg(rank_col + d0 + t);
+      }
+    };
+    load_ranks(min(dy_begin, hi + 1 - kMeT));
+
+#pragma unroll 1
+    for (int hs = 0; hs < NSTG; ++hs) {
+    const int yst = yw0 + hs * (S / NSTG);                // frame row of staged window row 0
     __syncthreads();
     // ---- a1: stage 4 byte-shifted copies of the SA window ----
     // item = (window row, 16-byte chunk k): raw words 4k..4k+4 -> words 4k..4k+3
@@ -385,7 +428,7 @@ __global__ void __launch_bounds__(S_CT ? 128 : 256, S_CT ? FEVES_ME_MINB : 2) me
       const bool vec_ok = P.vec_ok;
       for (int item = threadIdx.x; item < win_rows * chunks; item += blockDim.x) {
         const int row = item / chunks, k = item - row * chunks;
-        const int x = xw0 + 16 * k, y = min(max(yw0 + row, 0), P.H - 1);
+        const int x = xw0 + 16 * k, y = min(max(yst + row, 0), P.H - 1);
         uint32_t w[5];
         if (vec_ok && x >= 0 && x + 20 <= P.W) {
           const uint8_t* src = rf + (size_t)y * P.W + x;
@@ -411,25 +454,7 @@ __global__ void __launch_bounds__(S_CT ? 128 : 256, S_CT ? FEVES_ME_MINB : 2) me
     }
     __syncthreads();
 
-    uint32_t M[kNPart];
-#pragma unroll
-    for (int p = 0; p < kNPart; ++p) M[p] = 0xffffffffu;
-
-    // the lane's rank column (dy contiguous): with a compile-time S (a multiple of 4)
-    // every chunk start dy0 + R is a multiple of 4, so a chunk's ranks are ONE LDG.128
-    const uint32_t* rank_col = P.rank_tab + off * me_rank_pitch(S) + R;
-    uint32_t rank_next[kMeT];
-    auto load_ranks = [&](int d0) {
-      if (S_CT > 0 && kMeT == 4) {
-        const uint4 v = __ldg(reinterpret_cast<const uint4*>(rank_col + d0));
-        rank_next[0] = v.x; rank_next[1] = v.y; rank_next[2] = v.z; rank_next[3] = v.w;
-      } else {
-#pragma unroll
-        for (int t = 0; t < kMeT; ++t) rank_next[t] = __ldg(rank_col + d0 + t);
-      }
-    };
-    load_ranks(min(dy_begin, hi + 1 - kMeT));
-    for (int c = 0; c < DYL; c += kMeT) {
+    for (int c = hs * (DYL / NSTG); c < (hs + 1) * (DYL / NSTG); c += kMeT) {
       const int dy0 = min(dy_begin + c, hi + 1 - kMeT);   // clamped chunk: duplicates are harmless
       uint32_t rank[kMeT];
 #pragma unroll
@@ -437,7 +462,7 @@ __global__ void __launch_bounds__(S_CT ? 128 : 256, S_CT ? FEVES_ME_MINB : 2) me
       {                                                   // prefetch the next chunk's ranks
         load_ranks(min(dy_begin + c + kMeT, hi + 1 - kMeT));
       }
-      const uint32_t* wrow = wbase + (dy0 + R) * PW;
+      const uint32_t* wrow = wbase + (dy0 + R - hs * (S / NSTG)) * PW;
 
       uint32_t acc[kMeT][4];
       RowState st[kMeT];
@@ -481,19 +506,43 @@ __global__ void __launch_bounds__(S_CT ? 128 : 256, S_CT ? FEVES_ME_MINB : 2) me
       }
     }
 
+    if (QUAD && hs == 0) {                                // end of the dy < 0 quadrant half
+#pragma unroll
+      for (int p = 0; p < kNPart; ++p) {
+        const uint32_t v = __reduce_min_sync(0xffffffffu, M[p]);
+        if (lane == 0) red[(warp * NH) * kNPart + p] = v;
+        M[p] = 0xffffffffu;
+      }
+    }
+    }   // hs
+
     // ---- a4: warp min (CREDUX), then CTA min through shared memory ----
 #pragma unroll
     for (int p = 0; p < kNPart; ++p) {
       const uint32_t v = __reduce_min_sync(0xffffffffu, M[p]);
-      if (lane == 0) red[warp * kNPart + p] = v;
+      if (lane == 0) red[(warp * NH + NH - 1) * kNPart + p] = v;
     }
     __syncthreads();
     for (int p = threadIdx.x; p < kNPart; p += blockDim.x) {
-      uint32_t k = red[p];
-      for (int w = 1; w < nwarps; ++w) k = min(k, red[w * kNPart + p]);
-      const uint32_t rk = SumKeys<S_CT, KSH>::value ? (k & 0xffffu) >> part_log2n(p) : k & ((1u << KSH) - 1u);
+      uint32_t k, rk, sad;
+      if (QUAD) {                                            // (SAD, global dense rank), 30 bits
+        k = 0xffffffffu;
+        for (int w = 0; w < nwarps; ++w)
+          for (int hf = 0; hf < 2; ++hf) {
+            const uint32_t v = red[(w * 2 + hf) * kNPart + p];
+            const int q = 2 * hf + (w >= nwarps / 2 ? 1 : 0);   // quadrant: dy half, dx half
+            const uint32_t g = __ldg(P.glob_tab + q * 4096 + ((v & 0xffffu) >> part_log2n(p)));
+            k = min(k, ((v >> 16) << 14) | g);
+          }
+        rk = k & 0x3fffu;
+        sad = k >> 14;
+      } else {
+        k = red[p];
+        for (int w = 1; w < nwarps; ++w) k = min(k, red[w * kNPart + p]);
+        rk = SumKeys<S_CT, KSH>::value ? (k & 0xffffu) >> part_log2n(p) : k & ((1u << KSH) - 1u);
+        sad = k >> KSH;                                      // J = SAD + lambda*R(mv) (G18)
+      }
       const uint32_t mv = __ldg(P.inv_tab + rk);
-      uint32_t sad = k >> KSH;                               // J = SAD + lambda*R(mv) (G18)
       if (KSH != 16)
         sad -= (uint32_t)(P.lambda * (se_bits(4 * (int)(int16_t)(mv & 0xffffu)) + se_bits(4 * (int)(int16_t)(mv >> 16))));
       const size_t o = ((size_t)(blockIdx.y * P.mb_cols + mbx) * P.rf_stride + ref) * kNPart + p;

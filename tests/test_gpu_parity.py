@@ -150,9 +150,9 @@ def test_encode_frame_equals_separate_calls(feves):
     me.close()
 
 
-@pytest.mark.parametrize("fused", [True, False])
-def test_stream_fused_and_unfused_agree(feves, orc, fused):
-    W, H, S, n_rf = 96, 64, 32, 2
+@pytest.mark.parametrize("fused,S", [(True, 32), (False, 32), (True, 128), (False, 128)])
+def test_stream_fused_and_unfused_agree(feves, orc, fused, S):
+    W, H, n_rf = 96, 64, 2
     frames = [gen_noise(W, H, t, 17) for t in range(4)]
     me = feves.MotionEstimator(W, H, S, n_rf)
     me.set_fused(fused)
@@ -327,7 +327,7 @@ def test_stream_host_pipeline_many_frames(feves, orc):
     me.close()
 
 
-@pytest.mark.parametrize("lam,S", [(4, 16), (25, 32), (200, 8)])
+@pytest.mark.parametrize("lam,S", [(4, 16), (25, 32), (200, 8), (9, 128)])
 def test_rate_term_me_sme_and_mode_decision(feves, orc, lam, S):
     """f4 (G18) and f2 (O4) on the GPU path vs the oracle, bit-exact"""
     W, H, n_rf = 80, 48, 2
