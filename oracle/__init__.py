@@ -66,6 +66,8 @@ def lib():
             getattr(L, fn).argtypes = [P, i, i, i, i]
             getattr(L, fn).restype = i
         L.oracle_spiral_rank.argtypes = [i, i]
+        L.oracle_spiral_candidates.argtypes = [i, i, P, P]
+        L.oracle_spiral_candidates.restype = i
         L.oracle_partition_geom.argtypes = [i, P]
         L.oracle_num_threads.restype = i
         _lib = L
@@ -99,6 +101,14 @@ def partition_geom(p: int):
 
 def spiral_rank(dx: int, dy: int) -> int:
     return lib().oracle_spiral_rank(dx, dy)
+
+
+def spiral_candidates(S: int, sa_inclusive: bool = False):
+    """The SA's candidates (dx, dy) in the order O1 visits them (G1, G4)."""
+    n = (S + int(sa_inclusive)) ** 2
+    dx, dy = np.zeros(n, np.int32), np.zeros(n, np.int32)
+    assert lib().oracle_spiral_candidates(S, int(sa_inclusive), _ptr(dx), _ptr(dy)) == n
+    return list(zip(dx.tolist(), dy.tolist()))
 
 
 def all_mbs(W: int, H: int, row_begin: int = 0, row_end: int | None = None):

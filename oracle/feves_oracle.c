@@ -104,6 +104,12 @@ static int spiral_candidates(int S, int sa_inclusive, int *odx, int *ody)
     return n;
 }
 
+/* the SA's candidates in the order O1 visits them (exported for the key-table test) */
+int oracle_spiral_candidates(int S, int sa_inclusive, int *odx, int *ody)
+{
+    return spiral_candidates(S, sa_inclusive, odx, ody);
+}
+
 /* rank of (dx,dy) in the unrestricted spiral, by enumeration (P10 pins it) */
 int oracle_spiral_rank(int dx, int dy)
 {

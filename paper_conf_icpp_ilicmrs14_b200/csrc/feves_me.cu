@@ -138,25 +138,28 @@ static int launch_status() {
 // with lambda = 0 this is the spiral rank and key = SAD * 2^16 + rank; with a rate
 // term J = SAD + lambda*R may exceed 16 bits, so key = J * 2^15 + rank (rank < 2^15
 // for S <= 128, J < 2^17 for lambda <= 2000).
-static int upload_key_table(me_ctx* c) {
-  const int Sc = c->S + c->inclusive, hi = Sc - 1 - c->R;   // candidates per axis, dx,dy in [-R, hi]
-  c->kshift = c->lambda ? 15 : 16;
-  c->kmul = 1u << c->kshift;
+// Host-only construction of the three ME key tables (no CUDA call; me_key_tables exposes it).
+// e: [Sc][Sp] key addends, [dx+R][dy+R]; inv: dense rank -> packed MV; glob: S = 128 quadrant map.
+static void build_key_tables(int S, int inclusive, int lambda, std::vector<uint32_t>& e, std::vector<uint32_t>& inv,
+                             std::vector<uint32_t>& glob) {
+  const int R = S / 2, Sc = S + inclusive, hi = Sc - 1 - R;   // candidates per axis, dx,dy in [-R, hi]
+  const uint32_t kmul = 1u << (lambda ? 15 : 16);
   const int Sp = me_rank_pitch(Sc);
-  std::vector<uint32_t> e((size_t)Sc * Sp, 0), inv((size_t)(c->S + 1) * (c->S + 1), 0);
+  e.assign((size_t)Sc * Sp, 0);
+  inv.assign((size_t)(S + 1) * (S + 1), 0);
+  glob.assign(4 * 4096, 0);
   // DENSE rank: the candidates of the SA numbered 0..Sc^2-1 in spiral order (G4).  It
   // orders candidates exactly as the spiral rank does, and < 4096 for S <= 64 is what
   // lets the ME kernel build parent keys as sums of child keys (me_fsbm.cuh, SumKeys).
   std::vector<std::pair<int, uint32_t>> order;
   order.reserve((size_t)Sc * Sc);
-  for (int dy = -c->R; dy <= hi; ++dy)
-    for (int dx = -c->R; dx <= hi; ++dx)
+  for (int dy = -R; dy <= hi; ++dy)
+    for (int dx = -R; dx <= hi; ++dx)
       order.emplace_back(spiral_rank_closed_form(dx, dy), (uint32_t)(uint16_t)dx | ((uint32_t)(uint16_t)dy << 16));
   std::sort(order.begin(), order.end());
   // S = 128, pure SAD: the ME kernel sums keys quadrant by quadrant (me_fsbm.cuh QuadKeys),
   // so its table holds the rank inside the candidate's quadrant, and glob maps it back
-  const bool quad = c->S == 128 && !c->inclusive && !c->lambda;
-  std::vector<uint32_t> glob(4 * 4096, 0);
+  const bool quad = S == 128 && !inclusive && !lambda;
   int qn[4] = {0, 0, 0, 0};
   for (size_t r = 0; r < order.size(); ++r) {
     const int dx = (int)(int16_t)(order[r].second & 0xffffu), dy = (int)(int16_t)(order[r].second >> 16);
@@ -166,10 +169,30 @@ static int upload_key_table(me_ctx* c) {
       glob[q * 4096 + qn[q]] = (uint32_t)r;
       key_rank = (uint32_t)qn[q]++;
     }
-    e[(size_t)(dx + c->R) * Sp + (dy + c->R)] =
-        (uint32_t)(c->lambda * (se_bits(4 * dx) + se_bits(4 * dy))) * c->kmul + key_rank;
+    e[(size_t)(dx + R) * Sp + (dy + R)] = (uint32_t)(lambda * (se_bits(4 * dx) + se_bits(4 * dy))) * kmul + key_rank;
     inv[r] = order[r].second;
   }
+}
+
+extern "C" int me_key_tables(int sa_range, int inclusive, int lambda, uint32_t* key_addend, uint32_t* inv,
+                             uint32_t* glob) {
+  if (sa_range < 4 || sa_range > 128 || (sa_range & 1) || (inclusive != 0 && inclusive != 1) || lambda < 0 ||
+      lambda > 2000 || !key_addend || !inv || !glob)
+    return ME_EINVAL;
+  std::vector<uint32_t> e, iv, g;
+  build_key_tables(sa_range, inclusive, lambda, e, iv, g);
+  std::copy(e.begin(), e.end(), key_addend);
+  std::copy(iv.begin(), iv.end(), inv);
+  std::copy(g.begin(), g.end(), glob);
+  return ME_OK;
+}
+
+static int upload_key_table(me_ctx* c) {
+  const int Sc = c->S + c->inclusive;
+  c->kshift = c->lambda ? 15 : 16;
+  c->kmul = 1u << c->kshift;
+  std::vector<uint32_t> e, inv, glob;
+  build_key_tables(c->S, c->inclusive, c->lambda, e, inv, glob);
   c->me_threads = me_threads(Sc);
   c->me_smem = (size_t)me_smem_words(Sc) * 4;
   c->me_smem_fused = (size_t)me_smem_words_fused(Sc, c->n_rf) * 4;
