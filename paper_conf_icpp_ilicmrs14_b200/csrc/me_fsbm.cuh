@@ -14,16 +14,18 @@
 //      is loaded once and reused by 4 candidates (19 rows for 4 candidates).
 //      The 16 CF rows of the MB live in 64 registers.  Each 4x4 SAD is 4
 //      chained VABSDIFF4.ACC (one instruction per 4 px, ALU pipe);
-//  a3  aggregation is done directly in KEY space on the FMA pipe:
-//      key(child) = sad<<16 | rank, key(parent) = IMAD(sad(other child), 2^16,
-//      key(child)) -- one IMAD per partition, no ALU op;
+//  a3  aggregation is done directly in KEY space on the FMA pipe: key(4x4) =
+//      sad<<16 | rank; S <= 64 (and S = 128 quadrant by quadrant): key(parent) =
+//      key(child a) + key(child b) with the dense rank (SumKeys, below); otherwise
+//      key(parent) = IMAD(sad(other child), 2^KSH, key(child)).  One IMAD per
+//      partition, no ALU op;
 //  a4  per partition a running minimum of keys; two candidates per 3-input
 //      VIMNMX3 (ALU).  key = SAD * 2^16 + spiral rank (G4) makes the argmin
 //      unique and independent of the reduction order.  Warp: CREDUX.MIN
 //      (__reduce_min_sync); CTA: shared memory; rank -> (dx,dy) by table.
 // Roofline: ALU pipe = 64 lanes/clk/SM for VABSDIFF4, VIMNMX3,
 // IADD3 (measured, profiles/r01/int_peaks.json); per MB-candidate 64
-// VABSDIFF4 + 20.5 VIMNMX3 on ALU, ~55 IMAD on FMA.
+// VABSDIFF4 + 20.5 VIMNMX3 on ALU, 41 IMAD on FMA (key-sum; 54 otherwise).
 #pragma once
 #include "common.cuh"
 
