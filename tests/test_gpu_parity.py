@@ -230,6 +230,31 @@ def test_full_size_sampled(feves, orc, name, n_random):
     me.close()
 
 
+@pytest.mark.parametrize("kind", ["tex", "flat", "noise"])
+def test_full_frame_1080p_s64_every_mb(feves, orc, kind):
+    """1080p, SA 64x64 (the bench's ME kernel), 1 RF: EVERY MB's 41 MVs/SADs (ME and SME) and the
+    whole SF equal the oracle -- not a sample (the oracle takes ~10 s on the box's cores)."""
+    cfg = CONFIGS["1080p_sa64_4rf"]
+    cf, rfs = make_workload(cfg, kind=kind)
+    rfs = rfs[:1]
+    me = feves.MotionEstimator(cfg.width, cfg.height, cfg.sa_range, 1)
+    tcf, trfs = _dev(cf), [_dev(r) for r in rfs]
+    sfs = [me.new_sf()]
+    (mvs, sads), (qmvs, qsads) = me.encode_frame(tcf, trfs, sfs, n_int=1, out_me=me.new_mvs())
+    torch.cuda.synchronize()
+    n = me.mb_rows * me.mb_cols
+    o_mvs, o_sads = orc.me(cf, rfs, cfg.sa_range)
+    np.testing.assert_array_equal(sads.cpu().numpy().reshape(n, 1, 41), o_sads)
+    np.testing.assert_array_equal(mvs.cpu().numpy().reshape(n, 1, 41, 2), o_mvs)
+    o_q, o_qs = orc.sme(cf, rfs, o_mvs)
+    np.testing.assert_array_equal(qsads.cpu().numpy().reshape(n, 1, 41), o_qs)
+    np.testing.assert_array_equal(qmvs.cpu().numpy().reshape(n, 1, 41, 2), o_q)
+    if kind == "tex":
+        pad, pitch, rows = orc.sf_layout(cfg.width, cfg.height, cfg.sa_range)
+        np.testing.assert_array_equal(sfs[0].cpu().numpy(), orc.int_planes(rfs[0], pad, pitch, rows))
+    me.close()
+
+
 def test_determinism(feves):
     cfg = CONFIGS["1080p_sa32"]
     cf, rfs = make_workload(cfg, kind="flat")
