@@ -472,6 +472,13 @@ def run_feves(args, cfg):
                          "frac": u["int_bytes"] * stripe_frac / (int_iso_clean_ms / 1e3) / 1e9 / pk.get("hbm_gbs", 6650.0)},
         "cpu_baseline": cpu,
     }
+    if sme_ms:   # SME against the same ALU roofline (its binding resource is L1 latency/wavefronts)
+        sme_px_s = u["sme_px"] * stripe_frac / (sme_ms / 1e3)
+        line["roofline_sme"] = {"bound": "alu", "kernel": "sme_refine_kernel", "timing": "in the step",
+                                "achieved": sme_px_s / 1e12, "peak": peak_px / 1e12, "unit": "Tpx-absdiff/s",
+                                "frac": sme_px_s / peak_px,
+                                "note": "latency / L1-data-pipe bound, not ALU (ncu: 76% of L1 data-pipe "
+                                        "wavefronts, 41% issue active; DESIGN.md §6)"}
     print(json.dumps(line), flush=True)
     if world > 1:
         dist.destroy_process_group()
