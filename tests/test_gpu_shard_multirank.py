@@ -111,7 +111,7 @@ def _peer_worker(rank, world, port, q, host_frames):
         dist.destroy_process_group()
 
 
-@pytest.mark.parametrize("world,host_frames", [(2, False), (3, True)])
+@pytest.mark.parametrize("world,host_frames", [(2, False), (3, True), (4, False)])
 def test_peer_stream_equals_single(world, host_frames):
     """PeerStream (SURVEY §8(e) fused exchange): frames pulled as stripe + halo rows from
     rank 0's IPC-exported slot, SME outputs stored straight into rank 0's IPC-exported
