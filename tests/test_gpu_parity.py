@@ -255,6 +255,29 @@ def test_full_frame_1080p_s64_every_mb(feves, orc, kind):
     me.close()
 
 
+def test_2160p_s128_every_mb_of_three_rows(feves, orc):
+    """2160p, SA 128x128 (quadrant key-sum, half-window staging), 1 RF: every MB of the top,
+    middle and bottom MB rows (720 MBs incl. both frame corners) equals the oracle, ME and SME."""
+    cfg = CONFIGS["2160p_sa128"]
+    cf, rfs = make_workload(cfg, kind="tex")
+    rfs = rfs[:1]
+    me = feves.MotionEstimator(cfg.width, cfg.height, cfg.sa_range, 1)
+    tcf, trfs = _dev(cf), [_dev(r) for r in rfs]
+    sfs = [me.new_sf()]
+    (mvs, sads), (qmvs, qsads) = me.encode_frame(tcf, trfs, sfs, n_int=1, out_me=me.new_mvs())
+    torch.cuda.synchronize()
+    n = me.mb_rows * me.mb_cols
+    rows = (0, me.mb_rows // 2, me.mb_rows - 1)
+    mbs = np.array([r * me.mb_cols + c for r in rows for c in range(me.mb_cols)], np.int32)
+    o_mvs, o_sads = orc.me(cf, rfs, cfg.sa_range, mb_list=mbs)
+    np.testing.assert_array_equal(sads.cpu().numpy().reshape(n, 1, 41)[mbs], o_sads)
+    np.testing.assert_array_equal(mvs.cpu().numpy().reshape(n, 1, 41, 2)[mbs], o_mvs)
+    o_q, o_qs = orc.sme(cf, rfs, o_mvs, mb_list=mbs)
+    np.testing.assert_array_equal(qsads.cpu().numpy().reshape(n, 1, 41)[mbs], o_qs)
+    np.testing.assert_array_equal(qmvs.cpu().numpy().reshape(n, 1, 41, 2)[mbs], o_q)
+    me.close()
+
+
 def test_determinism(feves):
     cfg = CONFIGS["1080p_sa32"]
     cf, rfs = make_workload(cfg, kind="flat")
