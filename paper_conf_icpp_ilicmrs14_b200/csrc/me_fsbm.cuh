@@ -476,13 +476,22 @@ __global__ void __launch_bounds__(S_CT ? 128 : 256, S_CT ? FEVES_ME_MINB : 2) me
         uint32_t w[4];
 #pragma unroll
         for (int b = 0; b < 4; ++b) w[b] = wrow[i * PW + b];
+        // all SADs of this RF row first (word-major), then the keys / folds of the candidates
+        // whose 4x4 block row it completes (measured 0.3% faster than candidate-major)
+#pragma unroll
+        for (int b = 0; b < 4; ++b)
+#pragma unroll
+          for (int t = 0; t < kMeT; ++t) {
+            const int r = i - t;                            // CF row paired with RF row i
+            if (r >= 0 && r < 16) {
+              const uint32_t cw[4] = {cfr[r].x, cfr[r].y, cfr[r].z, cfr[r].w};
+              acc[t][b] = vad4(cw[b], w[b], (r & 3) ? acc[t][b] : 0u);
+            }
+          }
 #pragma unroll
         for (int t = 0; t < kMeT; ++t) {
-          const int r = i - t;                              // CF row paired with RF row i
+          const int r = i - t;
           if (r >= 0 && r < 16) {
-            const uint32_t cw[4] = {cfr[r].x, cfr[r].y, cfr[r].z, cfr[r].w};
-#pragma unroll
-            for (int b = 0; b < 4; ++b) acc[t][b] = vad4(cw[b], w[b], (r & 3) ? acc[t][b] : 0u);
             if ((r & 3) == 3) {
               const int by = r >> 2;
               if (SumKeys<S_CT, KSH>::value) {
