@@ -58,6 +58,9 @@ def lib():
         L.oracle_satd_q.argtypes = [P, P, i, i, i, i, i, i, i, i]
         L.oracle_satd_q.restype = ctypes.c_long
         L.oracle_mode_decision.argtypes = [P, P, i, i, i, P]
+        L.oracle_me_pmv.argtypes = [P, P, i, i, i, i, i, i, P, i, P, i, P, P, i]
+        L.oracle_sme_pmv.argtypes = [P, P, i, i, i, i, i, P, i, P, i, P, P, P, i]
+        L.oracle_mode_decision_pmv.argtypes = [P, P, i, i, i, P, i, P]
         L.oracle_mv_bits.argtypes = [i, i]
         L.oracle_mv_bits.restype = i
         L.oracle_int_planes.argtypes = [P, i, i, i, i, i, i, i, P, i]
@@ -117,9 +120,19 @@ def all_mbs(W: int, H: int, row_begin: int = 0, row_end: int | None = None):
     return np.arange(row_begin * mb_cols, row_end * mb_cols, dtype=np.int32)
 
 
-def me(cf, rfs, sa_range: int, mb_list=None, sa_inclusive: bool = False, threads: int = 0, lam: int = 0):
-    """O1 (lam > 0: cost J = SAD + lam * R(mv), G18). Returns (mvs int16 [n_mb, n_rf, 41, 2],
-    sads uint16 [n_mb, n_rf, 41]) -- the SAD of the chosen MV."""
+def _pmv(pmv, n, n_rf):
+    """G21 predictor array int16 [n, n_rf, 2] (or None = the zero predictor)."""
+    if pmv is None:
+        return None
+    return np.ascontiguousarray(pmv, np.int16).reshape(n, n_rf, 2)
+
+
+def me(cf, rfs, sa_range: int, mb_list=None, sa_inclusive: bool = False, threads: int = 0, lam: int = 0,
+       pmv=None, max_pmv: int = 0):
+    """O1 (lam > 0: cost J = SAD + lam * R(mv - p), G18; pmv: integer-pel predictor p per
+    (frame MB, RF) [mb_rows * mb_cols, n_rf, 2], each component clamped to +-max_pmv, the SA
+    centred on p, G21). Returns (mvs int16 [n_mb, n_rf, 41, 2], sads uint16 [n_mb, n_rf, 41])
+    -- the SAD of the chosen MV."""
     cf = _u8(cf)
     rfs = [_u8(r) for r in rfs]
     H, W = cf.shape
@@ -127,15 +140,18 @@ def me(cf, rfs, sa_range: int, mb_list=None, sa_inclusive: bool = False, threads
     n = len(mb_list)
     mvs = np.zeros((n, len(rfs), N_PART, 2), np.int16)
     sads = np.zeros((n, len(rfs), N_PART), np.uint16)
-    rc = lib().oracle_me_rd(_ptr(cf), _ptr_array(rfs), W, H, sa_range, len(rfs), int(sa_inclusive), int(lam),
-                            _ptr(mb_list), n, _ptr(mvs), _ptr(sads), threads)
+    pm = _pmv(pmv, ((W + 15) // 16) * ((H + 15) // 16), len(rfs))
+    rc = lib().oracle_me_pmv(_ptr(cf), _ptr_array(rfs), W, H, sa_range, len(rfs), int(sa_inclusive), int(lam),
+                             None if pm is None else _ptr(pm), int(max_pmv),
+                             _ptr(mb_list), n, _ptr(mvs), _ptr(sads), threads)
     if rc != 0:
         raise ValueError("oracle_me: bad arguments")
     return mvs, sads
 
 
-def sme(cf, rfs, in_mvs, mb_list=None, threads: int = 0, lam: int = 0, satd: bool = False):
-    """O3 (lam > 0: cost J = D + lam * R(qmv), G18; satd: D = Hadamard SATD, G20).
+def sme(cf, rfs, in_mvs, mb_list=None, threads: int = 0, lam: int = 0, satd: bool = False,
+        pmv=None, max_pmv: int = 0):
+    """O3 (lam > 0: cost J = D + lam * R(qmv - 4p), G18, G21 (pmv as for me); satd: D = Hadamard SATD, G20).
     in_mvs int16 [n_mb, n_rf, 41, 2] full-pel. Returns (qmvs, distortions)."""
     cf = _u8(cf)
     rfs = [_u8(r) for r in rfs]
@@ -145,8 +161,10 @@ def sme(cf, rfs, in_mvs, mb_list=None, threads: int = 0, lam: int = 0, satd: boo
     in_mvs = np.ascontiguousarray(in_mvs, np.int16).reshape(n, len(rfs), N_PART, 2)
     qmvs = np.zeros((n, len(rfs), N_PART, 2), np.int16)
     sads = np.zeros((n, len(rfs), N_PART), np.uint16)
-    rc = lib().oracle_sme_ex(_ptr(cf), _ptr_array(rfs), W, H, len(rfs), int(lam), int(satd), _ptr(mb_list), n,
-                             _ptr(in_mvs), _ptr(qmvs), _ptr(sads), threads)
+    pm = _pmv(pmv, ((W + 15) // 16) * ((H + 15) // 16), len(rfs))
+    rc = lib().oracle_sme_pmv(_ptr(cf), _ptr_array(rfs), W, H, len(rfs), int(lam), int(satd),
+                              None if pm is None else _ptr(pm), int(max_pmv), _ptr(mb_list), n,
+                              _ptr(in_mvs), _ptr(qmvs), _ptr(sads), threads)
     if rc != 0:
         raise ValueError("oracle_sme: bad arguments")
     return qmvs, sads
@@ -163,13 +181,16 @@ def mv_bits(qx: int, qy: int) -> int:
     return lib().oracle_mv_bits(qx, qy)
 
 
-def mode_decision(qmvs, sads, lam: int):
-    """O4: per MB [mb_type, sub_type x4, ref per 8x8 x4, cost] int32 [n_mb, 10]."""
+def mode_decision(qmvs, sads, lam: int, pmv=None, max_pmv: int = 0):
+    """O4: per MB [mb_type, sub_type x4, ref per 8x8 x4, cost] int32 [n_mb, 10].
+    pmv (G21): [n_mb, n_rf, 2] predictor of each listed MB; J uses R(qmv - 4p)."""
     qmvs = np.ascontiguousarray(qmvs, np.int16)
     sads = np.ascontiguousarray(sads, np.uint16)
     n, n_rf = sads.shape[0], sads.shape[1]
     out = np.zeros((n, 10), np.int32)
-    if lib().oracle_mode_decision(_ptr(qmvs), _ptr(sads), n, n_rf, int(lam), _ptr(out)) != 0:
+    pm = _pmv(pmv, n, n_rf)
+    if lib().oracle_mode_decision_pmv(_ptr(qmvs), _ptr(sads), n, n_rf, int(lam), None if pm is None else _ptr(pm),
+                                      int(max_pmv), _ptr(out)) != 0:
         raise ValueError("oracle_mode_decision: bad arguments")
     return out
 

@@ -157,10 +157,39 @@ int oracle_mv_bits(int qx, int qy) { return se_bits(qx) + se_bits(qy); }
  *   out_mvs [n_mb][n_rf][41][2] int16 (dx, dy) full-pel
  *   out_sads[n_mb][n_rf][41]    uint16
  * Returns 0, or -1 on bad arguments.                                      */
+/* G21 (SURVEY §8 f4 "predicted-MV centre"): an optional integer-pel MV predictor
+ * p per (MB, RF), supplied by the caller (pmv[(mb * n_rf + r) * 2 + {0,1}], mb =
+ * the frame MB index mby * mb_cols + mbx; NULL = the zero predictor of G2), each
+ * component clamped to [-max_pmv, max_pmv].  The SA is centred on p: candidates
+ * mv = p + (dx, dy) over the same (dx, dy) set and spiral order (G1, G4), and the
+ * rate term is R(mv - p) on the quarter-pel MV difference, as in JM's motion cost
+ * lambda * R(mv - pmv).                                                   */
+int oracle_me_pmv(const uint8_t *cf, const uint8_t *const *rfs, int W, int H,
+                  int S, int n_rf, int sa_inclusive, int lambda,
+                  const int16_t *pmv, int max_pmv,
+                  const int32_t *mb_list, int n_mb,
+                  int16_t *out_mvs, uint16_t *out_sads, int n_threads);
+
+static int clamp_pmv(const int16_t *pmv, int max_pmv, size_t idx, int comp)
+{
+    if (!pmv) return 0;
+    return clampi(pmv[2 * idx + comp], -max_pmv, max_pmv);
+}
+
 int oracle_me_rd(const uint8_t *cf, const uint8_t *const *rfs, int W, int H,
                  int S, int n_rf, int sa_inclusive, int lambda,
                  const int32_t *mb_list, int n_mb,
                  int16_t *out_mvs, uint16_t *out_sads, int n_threads)
+{
+    return oracle_me_pmv(cf, rfs, W, H, S, n_rf, sa_inclusive, lambda, NULL, 0, mb_list, n_mb,
+                         out_mvs, out_sads, n_threads);
+}
+
+int oracle_me_pmv(const uint8_t *cf, const uint8_t *const *rfs, int W, int H,
+                  int S, int n_rf, int sa_inclusive, int lambda,
+                  const int16_t *pmv, int max_pmv,
+                  const int32_t *mb_list, int n_mb,
+                  int16_t *out_mvs, uint16_t *out_sads, int n_threads)
 {
     if (W <= 0 || H <= 0 || S < 2 || (S & 1) || n_rf < 1) return -1;
     int mb_cols = (W + 15) / 16;
@@ -176,13 +205,15 @@ int oracle_me_rd(const uint8_t *cf, const uint8_t *const *rfs, int W, int H,
         int mbx = mb_list[i] % mb_cols, mby = mb_list[i] / mb_cols;
         for (int r = 0; r < n_rf; ++r) {
             const uint8_t *rf = rfs[r];
+            size_t pi = (size_t)mb_list[i] * n_rf + r;
+            int px = clamp_pmv(pmv, max_pmv, pi, 0), py = clamp_pmv(pmv, max_pmv, pi, 1);   /* G21 */
             for (int p = 0; p < 41; ++p) {
                 int ox, oy, w, h;
                 partition_geom(p, &ox, &oy, &w, &h);
                 int x0 = 16 * mbx + ox, y0 = 16 * mby + oy;
                 long best = -1, best_sad = 0; int bdx = 0, bdy = 0;
                 for (int c = 0; c < nc; ++c) {          /* spiral order, strict < */
-                    int dx = cdx[c], dy = cdy[c];
+                    int dx = px + cdx[c], dy = py + cdy[c];      /* mv = p + SA offset (G21) */
                     long sad = 0;
                     for (int j = 0; j < h; ++j)
                         for (int ii = 0; ii < w; ++ii) {
@@ -190,7 +221,7 @@ int oracle_me_rd(const uint8_t *cf, const uint8_t *const *rfs, int W, int H,
                             int b = ref_px(rf, W, H, x0 + ii + dx, y0 + j + dy);
                             sad += a > b ? a - b : b - a;
                         }
-                    long cost = sad + (long)lambda * se_bits(4 * dx) + (long)lambda * se_bits(4 * dy);
+                    long cost = sad + (long)lambda * se_bits(4 * (dx - px)) + (long)lambda * se_bits(4 * (dy - py));
                     if (best < 0 || cost < best) { best = cost; best_sad = sad; bdx = dx; bdy = dy; }
                 }
                 size_t o = ((size_t)i * n_rf + r) * 41 + p;
@@ -399,11 +430,25 @@ int oracle_sme_rd(const uint8_t *cf, const uint8_t *const *rfs, int W, int H, in
     return oracle_sme_ex(cf, rfs, W, H, n_rf, lambda, 0, mb_list, n_mb, in_mvs, out_qmvs, out_sads, n_threads);
 }
 
-/* metric: SAD (satd = 0, G13) or SATD (satd = 1, G20); outputs the metric value
- * (not the cost J) of the chosen vector */
+int oracle_sme_pmv(const uint8_t *cf, const uint8_t *const *rfs, int W, int H, int n_rf, int lambda, int satd,
+                   const int16_t *pmv, int max_pmv,
+                   const int32_t *mb_list, int n_mb, const int16_t *in_mvs,
+                   int16_t *out_qmvs, uint16_t *out_sads, int n_threads);
+
 int oracle_sme_ex(const uint8_t *cf, const uint8_t *const *rfs, int W, int H, int n_rf, int lambda, int satd,
                   const int32_t *mb_list, int n_mb, const int16_t *in_mvs,
                   int16_t *out_qmvs, uint16_t *out_sads, int n_threads)
+{
+    return oracle_sme_pmv(cf, rfs, W, H, n_rf, lambda, satd, NULL, 0, mb_list, n_mb, in_mvs, out_qmvs, out_sads,
+                          n_threads);
+}
+
+/* metric: SAD (satd = 0, G13) or SATD (satd = 1, G20); outputs the metric value
+ * (not the cost J) of the chosen vector.  pmv (G21): rate term R(v - 4p). */
+int oracle_sme_pmv(const uint8_t *cf, const uint8_t *const *rfs, int W, int H, int n_rf, int lambda, int satd,
+                   const int16_t *pmv, int max_pmv,
+                   const int32_t *mb_list, int n_mb, const int16_t *in_mvs,
+                   int16_t *out_qmvs, uint16_t *out_sads, int n_threads)
 {
     if (W <= 0 || H <= 0 || n_rf < 1) return -1;
     int mb_cols = (W + 15) / 16;
@@ -419,24 +464,26 @@ int oracle_sme_ex(const uint8_t *cf, const uint8_t *const *rfs, int W, int H, in
                 partition_geom(p, &ox, &oy, &w, &h);
                 int x0 = 16 * mbx + ox, y0 = 16 * mby + oy;
                 size_t o = ((size_t)i * n_rf + r) * 41 + p;
+                size_t pi = (size_t)mb_list[i] * n_rf + r;
+                int qpx = 4 * clamp_pmv(pmv, max_pmv, pi, 0), qpy = 4 * clamp_pmv(pmv, max_pmv, pi, 1);   /* G21 */
                 int cx = 4 * in_mvs[2 * o], cy = 4 * in_mvs[2 * o + 1];
                 /* cost J = SADq + lambda * R(v) (G18; lambda = 0: pure SAD, G13) */
 #define DIST(vx, vy) (satd ? satd_q(cf, rfs[r], W, H, x0, y0, w, h, vx, vy) \
                            : sad_q(cf, rfs[r], W, H, x0, y0, w, h, vx, vy))
                 long bsad = DIST(cx, cy);
-                long best = bsad + (long)lambda * (se_bits(cx) + se_bits(cy));
+                long best = bsad + (long)lambda * (se_bits(cx - qpx) + se_bits(cy - qpy));
                 int bx = cx, by = cy;
                 for (int k = 0; k < 8; ++k) {                     /* half-pel ring */
                     int vx = cx + 2 * ring1[k][0], vy = cy + 2 * ring1[k][1];
                     long s = DIST(vx, vy);
-                    long j = s + (long)lambda * (se_bits(vx) + se_bits(vy));
+                    long j = s + (long)lambda * (se_bits(vx - qpx) + se_bits(vy - qpy));
                     if (j < best) { best = j; bsad = s; bx = vx; by = vy; }
                 }
                 int qx = bx, qy = by;
                 for (int k = 0; k < 8; ++k) {                     /* quarter-pel ring */
                     int vx = qx + ring1[k][0], vy = qy + ring1[k][1];
                     long s = DIST(vx, vy);
-                    long j = s + (long)lambda * (se_bits(vx) + se_bits(vy));
+                    long j = s + (long)lambda * (se_bits(vx - qpx) + se_bits(vy - qpy));
                     if (j < best) { best = j; bsad = s; bx = vx; by = vy; }
                 }
 #undef DIST
@@ -470,8 +517,18 @@ int oracle_sme(const uint8_t *cf, const uint8_t *const *rfs, int W, int H, int n
  * order (lowest index wins ties).  With lambda = 0 the P8x8/4x4 choice never
  * loses (pin P4), so the decision is only informative with a rate term.
  * out[n_mb][10]: mb_type, sub_type[4] (-1 unless P8x8), ref per 8x8 quadrant [4], cost. */
+int oracle_mode_decision_pmv(const int16_t *qmvs, const uint16_t *sads, int n_mb, int n_rf, int lambda,
+                             const int16_t *pmv, int max_pmv, int32_t *out);
+
 int oracle_mode_decision(const int16_t *qmvs, const uint16_t *sads, int n_mb, int n_rf, int lambda,
                          int32_t *out)
+{
+    return oracle_mode_decision_pmv(qmvs, sads, n_mb, n_rf, lambda, NULL, 0, out);
+}
+
+/* pmv (G21): pmv[(i * n_rf + r) * 2 + {0,1}] for the i-th MB of the arrays; J uses R(qmv - 4p) */
+int oracle_mode_decision_pmv(const int16_t *qmvs, const uint16_t *sads, int n_mb, int n_rf, int lambda,
+                             const int16_t *pmv, int max_pmv, int32_t *out)
 {
     if (n_mb < 0 || n_rf < 1 || n_rf > 16) return -1;
     for (int i = 0; i < n_mb; ++i) {
@@ -479,7 +536,9 @@ int oracle_mode_decision(const int16_t *qmvs, const uint16_t *sads, int n_mb, in
         for (int r = 0; r < n_rf; ++r)
             for (int p = 0; p < 41; ++p) {
                 size_t o = ((size_t)i * n_rf + r) * 41 + p;
-                J[r][p] = (long)sads[o] + (long)lambda * (se_bits(qmvs[2 * o]) + se_bits(qmvs[2 * o + 1]));
+                size_t pi = (size_t)i * n_rf + r;
+                int qpx = 4 * clamp_pmv(pmv, max_pmv, pi, 0), qpy = 4 * clamp_pmv(pmv, max_pmv, pi, 1);
+                J[r][p] = (long)sads[o] + (long)lambda * (se_bits(qmvs[2 * o] - qpx) + se_bits(qmvs[2 * o + 1] - qpy));
             }
         long best = -1; int bt = 0, st[4] = {-1, -1, -1, -1}, rq[4] = {0, 0, 0, 0};
         /* 16x16 */

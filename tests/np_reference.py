@@ -276,3 +276,39 @@ def sme_satd(cf, rfs, mvs, S, lam=0):
                 qmvs[o, r, p] = bv
                 out[o, r, p] = bd
     return qmvs, out
+
+
+# ---------------------------------------------------- G21 predicted-MV centre --
+
+def me_pmv(cf, rfs, S, lam, pmv, max_pmv):
+    """brute force with an integer-pel predictor p per (MB, RF), clamped to +-max_pmv:
+    candidates p + (dx, dy), lexicographic (SAD + lam*R(4(mv - p)), rank(dx, dy)) minimum"""
+    H, W = cf.shape
+    R = S // 2
+    mbc, mbr = -(-W // 16), -(-H // 16)
+    Wp, Hp = 16 * mbc, 16 * mbr
+    cfp = _edge(cf, ((0, Hp - H), (0, Wp - W)))
+    m = R + 1 + max_pmv
+    d = np.arange(-R, R)
+    DX, DY = np.meshgrid(d, d)
+    rank = rank_closed_form(DX, DY).ravel()
+    rate = np.array([lam * (se_bits(4 * x) + se_bits(4 * y)) for x, y in zip(DX.ravel(), DY.ravel())])
+    pmv = np.clip(np.asarray(pmv, np.int64).reshape(mbr * mbc, len(rfs), 2), -max_pmv, max_pmv)
+    parts = partitions()
+    mvs = np.zeros((mbr * mbc, len(rfs), 41, 2), np.int16)
+    sads = np.zeros((mbr * mbc, len(rfs), 41), np.uint16)
+    for r, rf in enumerate(rfs):
+        rfp = _edge(rf, ((m, m + Hp - H), (m, m + Wp - W)))
+        for o in range(mbr * mbc):
+            mby, mbx = divmod(o, mbc)
+            px, py = int(pmv[o, r, 0]), int(pmv[o, r, 1])
+            for p, (ox, oy, w, h) in enumerate(parts):
+                x0, y0 = 16 * mbx + ox, 16 * mby + oy
+                blk = cfp[y0:y0 + h, x0:x0 + w]
+                cand = np.array([np.abs(blk - rfp[y0 + py + dy + m:y0 + py + dy + m + h,
+                                                  x0 + px + dx + m:x0 + px + dx + m + w]).sum()
+                                 for dy, dx in zip(DY.ravel(), DX.ravel())])
+                best = np.lexsort((rank, cand + rate))[0]
+                mvs[o, r, p] = (px + DX.ravel()[best], py + DY.ravel()[best])
+                sads[o, r, p] = cand[best]
+    return mvs, sads
