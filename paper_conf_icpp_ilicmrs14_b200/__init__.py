@@ -40,6 +40,9 @@ def lib():
         P, i = ctypes.c_void_p, ctypes.c_int
         L.me_create.restype = P
         L.me_create.argtypes = [i, i, i, i]
+        L.me_create_pmv.restype = P
+        L.me_create_pmv.argtypes = [i, i, i, i, i]
+        L.me_set_pmv.argtypes = [P, P]
         L.me_destroy.argtypes = [P]
         L.me_last_error.restype = i
         L.me_strerror.restype = ctypes.c_char_p
@@ -95,18 +98,20 @@ class MotionEstimator:
     [rows, mb_cols, n_rf, 41] uint16 (rows = the current MB-row stripe).
     """
 
-    def __init__(self, width: int, height: int, sa_range: int, n_rf: int, device=None):
+    def __init__(self, width: int, height: int, sa_range: int, n_rf: int, device=None, max_pmv: int = 0):
         if not torch.cuda.is_available():
             raise FevesError("no CUDA device: the FEVES path has no CPU fallback")
         self.device = torch.device("cuda", torch.cuda.current_device() if device is None else
                                    torch.device(device).index or 0)
         with torch.cuda.device(self.device):
             L = lib()
-            self._ctx = L.me_create(width, height, sa_range, n_rf)
+            self._ctx = L.me_create_pmv(width, height, sa_range, n_rf, max_pmv)
             if not self._ctx:
-                raise FevesError(f"me_create({width},{height},{sa_range},{n_rf}): "
+                raise FevesError(f"me_create_pmv({width},{height},{sa_range},{n_rf},{max_pmv}): "
                                  f"{L.me_strerror(L.me_last_error()).decode()}")
         self.width, self.height, self.sa_range, self.n_rf = width, height, sa_range, n_rf
+        self.max_pmv = max_pmv
+        self._pmv = None
         vals = [ctypes.c_int() for _ in range(5)]
         _check(lib().me_get_layout(self._ctx, *[ctypes.byref(v) for v in vals]))
         self.mb_cols, self.mb_rows, self.sf_pad, self.sf_pitch, self.sf_rows = [v.value for v in vals]
@@ -259,6 +264,17 @@ class MotionEstimator:
     def set_lambda(self, lam: int):
         """Rate term (f4, G18): ME and SME minimise SAD + lam * R(mv)."""
         self.set_option(self.OPT_LAMBDA, lam)
+
+    def set_pmv(self, pmv):
+        """MV predictor field (f4, G21; needs max_pmv > 0): int16 CUDA tensor
+        [mb_rows * mb_cols, n_rf, 2] integer-pel (x, y), or None = zero predictor.
+        The tensor is kept referenced: later calls read it."""
+        if pmv is not None:
+            if pmv.dtype != torch.int16 or not pmv.is_cuda or not pmv.is_contiguous() or \
+                    pmv.numel() != self.mb_rows * self.mb_cols * self.n_rf * 2:
+                raise FevesError("set_pmv: need a contiguous int16 CUDA tensor [mb_rows*mb_cols, n_rf, 2]")
+        _check(lib().me_set_pmv(self._ctx, None if pmv is None else pmv.data_ptr()))
+        self._pmv = pmv
 
     def mode_decision(self, qmvs, qsads, out=None):
         """Best H.264 P-MB configuration per MB (f2, me_mode_decision):

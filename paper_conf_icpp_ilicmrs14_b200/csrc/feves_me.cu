@@ -67,6 +67,8 @@ struct me_ctx {
   int lambda;            // G18 rate term (ME_OPT_LAMBDA); key = J * kmul + rank
   int satd;              // G20 SME distortion = Hadamard SATD (ME_OPT_SME_SATD)
   int inclusive;         // G1 alternative: candidates [-R, R]^2 (ME_OPT_SA_INCLUSIVE)
+  int max_pmv;           // G21: predictor clamp (me_create_pmv); > 0 routes ME to the runtime-S kernel
+  const int16_t* d_pmv;  // G21: predictor field (me_set_pmv), device, or null = zero predictor
   uint32_t kmul;
   int kshift;
   cudaStream_t sme_st;   // pipeline: SME stream
@@ -141,7 +143,7 @@ static int launch_status() {
 // Host-only construction of the three ME key tables (no CUDA call; me_key_tables exposes it).
 // e: [Sc][Sp] key addends, [dx+R][dy+R]; inv: dense rank -> packed MV; glob: S = 128 quadrant map.
 static void build_key_tables(int S, int inclusive, int lambda, std::vector<uint32_t>& e, std::vector<uint32_t>& inv,
-                             std::vector<uint32_t>& glob) {
+                             std::vector<uint32_t>& glob, bool allow_quad = true) {
   const int R = S / 2, Sc = S + inclusive, hi = Sc - 1 - R;   // candidates per axis, dx,dy in [-R, hi]
   const uint32_t kmul = 1u << (lambda ? 15 : 16);
   const int Sp = me_rank_pitch(Sc);
@@ -159,7 +161,7 @@ static void build_key_tables(int S, int inclusive, int lambda, std::vector<uint3
   std::sort(order.begin(), order.end());
   // S = 128, pure SAD: the ME kernel sums keys quadrant by quadrant (me_fsbm.cuh QuadKeys),
   // so its table holds the rank inside the candidate's quadrant, and glob maps it back
-  const bool quad = S == 128 && !inclusive && !lambda;
+  const bool quad = S == 128 && !inclusive && !lambda && allow_quad;
   int qn[4] = {0, 0, 0, 0};
   for (size_t r = 0; r < order.size(); ++r) {
     const int dx = (int)(int16_t)(order[r].second & 0xffffu), dy = (int)(int16_t)(order[r].second >> 16);
@@ -192,7 +194,7 @@ static int upload_key_table(me_ctx* c) {
   c->kshift = c->lambda ? 15 : 16;
   c->kmul = 1u << c->kshift;
   std::vector<uint32_t> e, inv, glob;
-  build_key_tables(c->S, c->inclusive, c->lambda, e, inv, glob);
+  build_key_tables(c->S, c->inclusive, c->lambda, e, inv, glob, c->max_pmv == 0);
   c->me_threads = me_threads(Sc);
   c->me_smem = (size_t)me_smem_words(Sc) * 4;
   c->me_smem_fused = (size_t)me_smem_words_fused(Sc, c->n_rf) * 4;
@@ -205,16 +207,22 @@ static int upload_key_table(me_ctx* c) {
 
 // ------------------------------------------------------------ lifetime ----
 extern "C" me_ctx* me_create(int width, int height, int sa_range, int n_rf) {
+  return me_create_pmv(width, height, sa_range, n_rf, 0);
+}
+
+extern "C" me_ctx* me_create_pmv(int width, int height, int sa_range, int n_rf, int max_pmv) {
   g_last_error = ME_EINVAL;
   if (width <= 0 || height <= 0 || width > 16384 || height > 16384) return nullptr;
   if (sa_range < 4 || sa_range > 128 || (sa_range & 1)) return nullptr;
+  if (max_pmv < 0 || max_pmv > 256 || (max_pmv > 0 && sa_range == 128)) return nullptr;
   if (n_rf < 1 || n_rf > kMaxRf) return nullptr;
   me_ctx* c = new (std::nothrow) me_ctx();
   if (!c) { g_last_error = ME_ENOMEM; return nullptr; }
   c->W = width; c->H = height; c->S = sa_range; c->R = sa_range / 2; c->n_rf = n_rf;
   c->mb_cols = (width + 15) / 16; c->mb_rows = (height + 15) / 16;
   c->row0 = 0; c->row1 = c->mb_rows;
-  c->sf_pad = ((c->R + 4 + 15) / 16) * 16;
+  c->max_pmv = max_pmv;   // G21: every MV stays within p +- R, |p| <= max_pmv -> SF margin covers it
+  c->sf_pad = ((c->R + max_pmv + 4 + 15) / 16) * 16;
   c->sf_pitch = 16 * c->mb_cols + 2 * c->sf_pad;
   c->sf_rows = 16 * c->mb_rows + 2 * c->sf_pad;
   if (cudaGetDevice(&c->device) != cudaSuccess) { delete c; g_last_error = ME_ECUDA; return nullptr; }
@@ -343,7 +351,7 @@ static void tmark(me_ctx* c, int i, cudaStream_t st) {
 // ME (and, when sfs != NULL, the fused SME of me_fsbm.cuh) over n_ref RFs
 static int launch_me(me_ctx* c, const uint8_t* cf, const uint8_t* const* rfs, int16_t* mvs, uint16_t* sads,
                      int n_ref, cudaStream_t st, const uint8_t* const* sfs = nullptr, int16_t* qmvs = nullptr,
-                     uint16_t* qsads = nullptr) {
+                     uint16_t* qsads = nullptr, int rf0 = 0) {
   MeParams P;
   memset(&P, 0, sizeof(P));
   P.cf = cf;
@@ -353,6 +361,8 @@ static int launch_me(me_ctx* c, const uint8_t* cf, const uint8_t* const* rfs, in
   P.rank_tab = c->d_rank; P.inv_tab = c->d_inv; P.glob_tab = c->d_glob;
   P.kmul = c->kmul; P.kshift = c->kshift; P.lambda = c->lambda;
   P.out_mvs = mvs; P.out_sads = sads;
+  P.pmv = c->d_pmv ? c->d_pmv + 2 * rf0 : nullptr;   // rf0: first RF of this launch (per-RF pipeline)
+  P.max_pmv = c->max_pmv;
   bool vec = (c->W % 16 == 0) && (c->R % 16 == 0);
   for (int k = 0; k < n_ref; ++k) vec = vec && ((reinterpret_cast<uintptr_t>(rfs[k]) & 15) == 0);
   P.vec_ok = vec ? 1 : 0;
@@ -375,7 +385,7 @@ static int launch_me(me_ctx* c, const uint8_t* cf, const uint8_t* const* rfs, in
     else if (c->lambda) me_fsbm_kernel<SS, false, 15><<<grid, c->me_threads, smem, st>>>(P); \
     else me_fsbm_kernel<SS, false><<<grid, c->me_threads, smem, st>>>(P);               \
   } while (0)
-  switch (c->inclusive ? 0 : c->S) {   // compile-time window geometry for the paper's SA sizes (Fig. 6a: 32..256)
+  switch (c->inclusive || c->max_pmv ? 0 : c->S) {   // compile-time window geometry for the paper's SA sizes (Fig. 6a: 32..256)
     case 16: FEVES_ME_LAUNCH(16); break;
     case 32: FEVES_ME_LAUNCH(32); break;
     case 64: FEVES_ME_LAUNCH(64); break;
@@ -397,8 +407,8 @@ static int launch_int(me_ctx* c, const uint8_t* rf, uint8_t* sf, cudaStream_t st
   if (c->row0 == 0 && c->row1 == c->mb_rows) {
     P.row_begin = 0; P.row_end = c->sf_rows;
   } else {   // stripe + halo: SME reads integer rows [16r0-R-1, 16r1+R-2]
-    P.row_begin = std::max(0, c->sf_pad + 16 * c->row0 - c->R - 4);
-    P.row_end = std::min(c->sf_rows, c->sf_pad + 16 * c->row1 + c->R + 4);
+    P.row_begin = std::max(0, c->sf_pad + 16 * c->row0 - c->R - c->max_pmv - 4);
+    P.row_end = std::min(c->sf_rows, c->sf_pad + 16 * c->row1 + c->R + c->max_pmv + 4);
   }
   const int groups = c->sf_pitch / 16;
   // interior groups: x0-4 >= 0 and x0+20 <= W with x0 = 16g - pad, rows 4-byte aligned
@@ -423,7 +433,8 @@ static int launch_int(me_ctx* c, const uint8_t* rf, uint8_t* sf, cudaStream_t st
 }
 
 static int launch_sme(me_ctx* c, const uint8_t* cf, const uint8_t* const* sfs, const int16_t* in_mvs,
-                      const uint16_t* in_sads, int16_t* out_qmvs, uint16_t* out_sads, int n_ref, cudaStream_t st) {
+                      const uint16_t* in_sads, int16_t* out_qmvs, uint16_t* out_sads, int n_ref, cudaStream_t st,
+                      int rf0 = 0) {
   SmeParams P;
   memset(&P, 0, sizeof(P));
   P.cf = cf;
@@ -436,6 +447,8 @@ static int launch_sme(me_ctx* c, const uint8_t* cf, const uint8_t* const* sfs, c
   P.n_rows = c->row1 - c->row0;
   P.groups = (c->mb_cols + 7) / 8;
   P.lambda = c->lambda;
+  P.pmv = c->d_pmv ? c->d_pmv + 2 * rf0 : nullptr;
+  P.max_pmv = c->max_pmv;
   P.pad = c->sf_pad; P.pitch = c->sf_pitch;
   P.plane = (size_t)c->sf_rows * c->sf_pitch;
   P.fence = is_peer_ptr(c, out_qmvs) || is_peer_ptr(c, out_sads);
@@ -483,11 +496,13 @@ static int run_me_sme(me_ctx* c, const uint8_t* cf, const uint8_t* const* rfs, c
   if (sf_ready && cudaStreamWaitEvent(c->sme_st, sf_ready, 0) != cudaSuccess) return launch_status();
   for (int k = 0; k < n_ref; ++k) {
     const size_t off = (size_t)k * kNPart;
-    if ((st = launch_me(c, cf, rfs + k, mvs + 2 * off, sads + off, 1, c->stream)) != ME_OK) return st;
+    if ((st = launch_me(c, cf, rfs + k, mvs + 2 * off, sads + off, 1, c->stream, nullptr, nullptr, nullptr, k)) != ME_OK)
+      return st;
     if (cudaEventRecord(c->ev_me[k], c->stream) != cudaSuccess ||
         cudaStreamWaitEvent(c->sme_st, c->ev_me[k], 0) != cudaSuccess)
       return launch_status();
-    if ((st = launch_sme(c, cf, sfs + k, mvs + 2 * off, sads + off, qmvs + 2 * off, qsads + off, 1, c->sme_st)) != ME_OK)
+    if ((st = launch_sme(c, cf, sfs + k, mvs + 2 * off, sads + off, qmvs + 2 * off, qsads + off, 1, c->sme_st, k)) !=
+        ME_OK)
       return st;
   }
   c->timing = saved;
@@ -542,7 +557,7 @@ extern "C" int me_encode_frame(me_ctx* c, const uint8_t* cf, const uint8_t* cons
   int st;
   for (int k = 0; k < n_int; ++k)
     if ((st = launch_int(c, rfs[k], sfs[k], c->stream)) != ME_OK) return st;
-  if (c->fuse && !c->lambda && !c->satd && !c->inclusive)   // ME with the SME fused (one launch; base reading only)
+  if (c->fuse && !c->lambda && !c->satd && !c->inclusive && !c->max_pmv)   // ME with the SME fused (one launch; base reading only)
     return launch_me(c, cf, rfs, out_mvs, out_sads, c->n_rf, c->stream, reinterpret_cast<const uint8_t* const*>(sfs),
                      out_qmvs, out_qsads);
   return run_me_sme(c, cf, rfs, reinterpret_cast<const uint8_t* const*>(sfs), mvs, sads, out_qmvs, out_qsads, c->n_rf,
@@ -701,9 +716,9 @@ extern "C" int me_stream_push(me_ctx* c, const uint8_t* cf, int cf_on_host, int1
     uint16_t* qs = (out_qsads && !out_on_host) ? out_qsads : (out_on_host ? c->d_qsads2[par] : c->d_qsads);
     // the device output buffer t & 1 is free once the download of push t-2 finished
     if (out_on_host && cudaStreamWaitEvent(c->stream, c->ev_down[par], 0) != cudaSuccess) return launch_status();
-    if (c->overlap && !c->pipeline && !(c->fuse && !c->lambda && !c->satd && !c->inclusive)) {
+    if (c->overlap && !c->pipeline && !(c->fuse && !c->lambda && !c->satd && !c->inclusive && !c->max_pmv)) {
       if ((st = push_overlapped(c, cur, rfs, sfs, new_rf, new_sf, qm, qs, n_ref, par)) != ME_OK) return st;
-    } else if (c->fuse && !c->lambda && !c->satd && !c->inclusive) {
+    } else if (c->fuse && !c->lambda && !c->satd && !c->inclusive && !c->max_pmv) {
       // fused: the SME of ref 0 reads SF(t-1), so INT(t-1) runs first on the same stream
       if ((st = launch_int(c, new_rf, new_sf, c->stream)) != ME_OK) return st;
       if ((st = launch_me(c, cur, rfs, nullptr, nullptr, n_ref, c->stream, sfs, qm, qs)) != ME_OK) return st;
@@ -893,6 +908,14 @@ extern "C" int me_ipc_close(me_ctx* c, void* dptr) {
 
 extern "C" int me_set_fused(me_ctx* c, int on) { return me_set_option(c, ME_OPT_FUSED_SME, on); }
 
+extern "C" int me_set_pmv(me_ctx* c, const int16_t* pmv) {
+  if (!c) return ME_EINVAL;
+  if (c->max_pmv == 0) return ME_ESTATE;               // the SF margin has no room for a predictor
+  if (pmv && !is_device_ptr(c, pmv)) return ME_EINVAL;
+  c->d_pmv = pmv;
+  return ME_OK;
+}
+
 extern "C" int me_mode_decision(me_ctx* c, const int16_t* qmvs, const uint16_t* qsads, int32_t* out_modes) {
   if (!c || !is_device_ptr(c, qmvs) || !is_device_ptr(c, qsads) || !is_device_ptr(c, out_modes)) return ME_EINVAL;
   ModeParams P;
@@ -902,6 +925,7 @@ extern "C" int me_mode_decision(me_ctx* c, const int16_t* qmvs, const uint16_t* 
   P.n_mb = (c->row1 - c->row0) * c->mb_cols;
   P.n_rf = c->n_rf;
   P.lambda = c->lambda;
+  P.pmv = c->d_pmv; P.max_pmv = c->max_pmv; P.mb0 = c->row0 * c->mb_cols;
   c->last_launches = 0;
   mode_decision_kernel<<<(P.n_mb + 127) / 128, 128, 0, c->stream>>>(P);
   c->last_launches++;

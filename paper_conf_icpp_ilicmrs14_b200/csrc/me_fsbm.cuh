@@ -53,6 +53,8 @@ struct MeParams {
   int kshift, lambda;
   int16_t* out_mvs;
   uint16_t* out_sads;
+  const int16_t* pmv;         // G21 predictor [frame MB][rf_stride][2] integer-pel (runtime-S kernel only), or null
+  int max_pmv;                // G21 clamp of each predictor component
   int vec_ok;                 // 16-byte aligned rows and window start: vector staging allowed
   // fused SME (template FUSE): SF of each RF, quarter-pel outputs
   const uint8_t* sf[kMaxRf];
@@ -399,6 +401,14 @@ __global__ void __launch_bounds__(S_CT ? 128 : 256, S_CT ? FEVES_ME_MINB : 2) me
 
   for (int ref = 0; ref < P.n_rf; ++ref) {
     const uint8_t* __restrict__ rf = P.rf[ref];
+    // G21: the SA of this (MB, RF) is centred on the clamped predictor p (runtime-S kernel only;
+    // the compile-time kernels never see a predictor, so their code is unchanged)
+    int pcx = 0, pcy = 0;
+    if (S_CT == 0 && P.pmv) {
+      const size_t pi = ((size_t)mby * P.mb_cols + mbx) * P.rf_stride + ref;
+      pcx = min(max((int)P.pmv[2 * pi], -P.max_pmv), P.max_pmv);
+      pcy = min(max((int)P.pmv[2 * pi + 1], -P.max_pmv), P.max_pmv);
+    }
     uint32_t M[kNPart];
 #pragma unroll
     for (int p = 0; p < kNPart; ++p) M[p] = 0xffffffffu;
@@ -420,17 +430,17 @@ __global__ void __launch_bounds__(S_CT ? 128 : 256, S_CT ? FEVES_ME_MINB : 2) me
 
 #pragma unroll 1
     for (int hs = 0; hs < NSTG; ++hs) {
-    const int yst = yw0 + hs * (S / NSTG);                // frame row of staged window row 0
+    const int yst = yw0 + pcy + hs * (S / NSTG);          // frame row of staged window row 0
     __syncthreads();
     // ---- a1: stage 4 byte-shifted copies of the SA window ----
     // item = (window row, 16-byte chunk k): raw words 4k..4k+4 -> words 4k..4k+3
     // of copies 0..3 (copy c word q = raw bytes [4q+c, 4q+c+4)), STS.128.
     {
       const int chunks = PW >> 2;
-      const bool vec_ok = P.vec_ok;
+      const bool vec_ok = P.vec_ok && (pcx & 15) == 0;
       for (int item = threadIdx.x; item < win_rows * chunks; item += blockDim.x) {
         const int row = item / chunks, k = item - row * chunks;
-        const int x = xw0 + 16 * k, y = min(max(yst + row, 0), P.H - 1);
+        const int x = xw0 + pcx + 16 * k, y = min(max(yst + row, 0), P.H - 1);
         uint32_t w[5];
         if (vec_ok && x >= 0 && x + 20 <= P.W) {
           const uint8_t* src = rf + (size_t)y * P.W + x;
@@ -553,9 +563,12 @@ __global__ void __launch_bounds__(S_CT ? 128 : 256, S_CT ? FEVES_ME_MINB : 2) me
         rk = SumKeys<S_CT, KSH>::value ? (k & 0xffffu) >> part_log2n(p) : k & ((1u << KSH) - 1u);
         sad = k >> KSH;                                      // J = SAD + lambda*R(mv) (G18)
       }
-      const uint32_t mv = __ldg(P.inv_tab + rk);
-      if (KSH != 16)
+      uint32_t mv = __ldg(P.inv_tab + rk);                   // SA offset (dx, dy)
+      if (KSH != 16)                                         // rate of the offset = R(mv - p) (G21)
         sad -= (uint32_t)(P.lambda * (se_bits(4 * (int)(int16_t)(mv & 0xffffu)) + se_bits(4 * (int)(int16_t)(mv >> 16))));
+      if (S_CT == 0 && P.pmv)                                // mv = p + offset (G21)
+        mv = (uint32_t)(uint16_t)((int)(int16_t)(mv & 0xffffu) + pcx) |
+             ((uint32_t)(uint16_t)((int)(int16_t)(mv >> 16) + pcy) << 16);
       const size_t o = ((size_t)(blockIdx.y * P.mb_cols + mbx) * P.rf_stride + ref) * kNPart + p;
       if (P.out_mvs) {
         reinterpret_cast<uint32_t*>(P.out_mvs)[o] = mv;

@@ -16,6 +16,8 @@ struct ModeParams {
   const uint16_t* sads;
   int32_t* out;             // [mb][10]: mb_type, sub_type[4], ref per 8x8 [4], cost
   int n_mb, n_rf, lambda;
+  const int16_t* pmv;       // G21 predictor [frame MB][n_rf][2] or null; MB i of the arrays = frame MB mb0 + i
+  int max_pmv, mb0;
 };
 
 __global__ void __launch_bounds__(128) mode_decision_kernel(const ModeParams P) {
@@ -26,7 +28,13 @@ __global__ void __launch_bounds__(128) mode_decision_kernel(const ModeParams P) 
     int j = P.sads[o];
     if (P.lambda) {
       const uint32_t mv = P.qmvs[o];
-      j += P.lambda * (se_bits((int)(int16_t)(mv & 0xffffu)) + se_bits((int)(int16_t)(mv >> 16)));
+      int qpx = 0, qpy = 0;                  // G21: rate against 4p
+      if (P.pmv) {
+        const size_t pi = ((size_t)(P.mb0 + i) * P.n_rf + r) * 2;
+        qpx = 4 * min(max((int)P.pmv[pi], -P.max_pmv), P.max_pmv);
+        qpy = 4 * min(max((int)P.pmv[pi + 1], -P.max_pmv), P.max_pmv);
+      }
+      j += P.lambda * (se_bits((int)(int16_t)(mv & 0xffffu) - qpx) + se_bits((int)(int16_t)(mv >> 16) - qpy));
     }
     return j;
   };

@@ -35,6 +35,8 @@ struct SmeParams {
   int pad, pitch;
   size_t plane;
   int lambda;                                         // G18 rate term (0 = pure SAD, G13)
+  const int16_t* pmv;                                 // G21 predictor [frame MB][rf_stride][2] or null
+  int max_pmv;
   int fence;                                          // outputs are peer memory (me_ipc_open): system fence at exit
   uint32_t k_hi;                                      // = kAvgHi (vavg4)
 };
@@ -252,7 +254,7 @@ __device__ __forceinline__ int mode_part(int bx, int by) {
 // RD = rate term (G18) compiled in; SATD = Hadamard distortion (G20) instead of SAD
 template <int MODE, int YG, int XMASK, bool RD, bool SATD>
 __device__ __forceinline__ void refine_mode(const SmeParams& P, const uint8_t* __restrict__ sf, size_t o, int bx,
-                                            int xs, int ys0, bool writer) {
+                                            int xs, int ys0, bool writer, int qpx, int qpy) {
   constexpr int NG = 4 / YG;           // partitions (block groups) inside this lane's strip
   // The groups are refined one after the other (latency-bound kernel: fewer live
   // registers -> more resident warps beats the ILP of refining all NG at once).
@@ -291,7 +293,7 @@ __device__ __forceinline__ void refine_mode(const SmeParams& P, const uint8_t* _
         s += strip_block_dist<SATD>(sf, P.plane, P.pitch, P.pad, xs, yg + 4 * j, bvx, bvy, cf + 4 * j);
       best = xsum<XMASK>(s);
     }
-    if (RD) best += P.lambda * (se_bits(bvx) + se_bits(bvy));   // J at the centre
+    if (RD) best += P.lambda * (se_bits(bvx - qpx) + se_bits(bvy - qpy));   // J at the centre
     // ---- half stage ----
     {
       const int ox = bvx, oy = bvy;
@@ -314,7 +316,7 @@ __device__ __forceinline__ void refine_mode(const SmeParams& P, const uint8_t* _
       for (int k = 0; k < 8; ++k) {                 // spiral order, strict < (G14)
         const int vx = ox + 2 * c_ring1[k][0], vy = oy + 2 * c_ring1[k][1];
         uint32_t t = xsum<XMASK>(sad[k]);
-        if (RD) t += P.lambda * (se_bits(vx) + se_bits(vy));
+        if (RD) t += P.lambda * (se_bits(vx - qpx) + se_bits(vy - qpy));
         if (t < best) { best = t; bvx = vx; bvy = vy; }
       }
     }
@@ -366,13 +368,13 @@ __device__ __forceinline__ void refine_mode(const SmeParams& P, const uint8_t* _
       for (int k = 0; k < 8; ++k) {             // spiral order, strict < (G14)
         const int vx = ox + c_ring1[k][0], vy = oy + c_ring1[k][1];
         uint32_t t = xsum<XMASK>(qs[k]);
-        if (RD) t += P.lambda * (se_bits(vx) + se_bits(vy));
+        if (RD) t += P.lambda * (se_bits(vx - qpx) + se_bits(vy - qpy));
         if (t < best) { best = t; bvx = vx; bvy = vy; }
       }
     }
     if (writer && (bx & XMASK) == 0) {     // partition leader lane writes
       P.out_qmvs[o + p] = (uint32_t)(uint16_t)bvx | ((uint32_t)(uint16_t)bvy << 16);
-      const uint32_t d = best - (RD ? P.lambda * (se_bits(bvx) + se_bits(bvy)) : 0);
+      const uint32_t d = best - (RD ? P.lambda * (se_bits(bvx - qpx) + se_bits(bvy - qpy)) : 0);
       P.out_sads[o + p] = (uint16_t)min(d, 65535u);        // SATD can exceed 16 bits (G20)
     }
   }
@@ -398,14 +400,20 @@ __global__ void __launch_bounds__(128, FEVES_SME_MINB) sme_refine_kernel(const S
   const int xs = 16 * mbx + 4 * bx, ys0 = 16 * mby;
   const uint8_t* __restrict__ sf = P.sf[ref];
   const size_t o = ((size_t)(mrow * P.mb_cols + mbx) * P.rf_stride + ref) * kNPart;
+  int qpx = 0, qpy = 0;                              // G21: rate against 4p (RD only)
+  if (RD && P.pmv) {
+    const size_t pi = ((size_t)mby * P.mb_cols + mbx) * P.rf_stride + ref;
+    qpx = 4 * min(max((int)P.pmv[2 * pi], -P.max_pmv), P.max_pmv);
+    qpy = 4 * min(max((int)P.pmv[2 * pi + 1], -P.max_pmv), P.max_pmv);
+  }
   switch (blockIdx.y) {   // one mode per warp: 7x the independent warps (the kernel is latency-bound)
-    case 0: refine_mode<0, 4, 3, RD, SATD>(P, sf, o, bx, xs, ys0, writer); break;   // 16x16
-    case 1: refine_mode<1, 2, 3, RD, SATD>(P, sf, o, bx, xs, ys0, writer); break;   // 16x8
-    case 2: refine_mode<2, 4, 1, RD, SATD>(P, sf, o, bx, xs, ys0, writer); break;   // 8x16
-    case 3: refine_mode<3, 2, 1, RD, SATD>(P, sf, o, bx, xs, ys0, writer); break;   // 8x8
-    case 4: refine_mode<4, 1, 1, RD, SATD>(P, sf, o, bx, xs, ys0, writer); break;   // 8x4
-    case 5: refine_mode<5, 2, 0, RD, SATD>(P, sf, o, bx, xs, ys0, writer); break;   // 4x8
-    default: refine_mode<6, 1, 0, RD, SATD>(P, sf, o, bx, xs, ys0, writer); break;  // 4x4
+    case 0: refine_mode<0, 4, 3, RD, SATD>(P, sf, o, bx, xs, ys0, writer, qpx, qpy); break;   // 16x16
+    case 1: refine_mode<1, 2, 3, RD, SATD>(P, sf, o, bx, xs, ys0, writer, qpx, qpy); break;   // 16x8
+    case 2: refine_mode<2, 4, 1, RD, SATD>(P, sf, o, bx, xs, ys0, writer, qpx, qpy); break;   // 8x16
+    case 3: refine_mode<3, 2, 1, RD, SATD>(P, sf, o, bx, xs, ys0, writer, qpx, qpy); break;   // 8x8
+    case 4: refine_mode<4, 1, 1, RD, SATD>(P, sf, o, bx, xs, ys0, writer, qpx, qpy); break;   // 8x4
+    case 5: refine_mode<5, 2, 0, RD, SATD>(P, sf, o, bx, xs, ys0, writer, qpx, qpy); break;   // 4x8
+    default: refine_mode<6, 1, 0, RD, SATD>(P, sf, o, bx, xs, ys0, writer, qpx, qpy); break;  // 4x4
   }
   if (P.fence) __threadfence_system();   // stores to another GPU's buffer are performed before the kernel ends
 }

@@ -65,3 +65,12 @@ def test_no_oracle_in_product_path():
             if f.endswith((".py", ".cu", ".cuh", ".h", ".cpp")):
                 txt = open(os.path.join(dirpath, f)).read()
                 assert "import oracle" not in txt and "from oracle" not in txt and "liboracle" not in txt, f
+
+
+@pytest.mark.parametrize("args", [(64, 64, 16, 1, -1), (64, 64, 16, 1, 257), (256, 256, 128, 1, 4)])
+def test_create_pmv_rejects_bad_arguments(feves_lib, args):
+    # G21: max_pmv in 0..256, and not with the S = 128 quadrant kernel; checked before any CUDA call
+    feves_lib.me_create_pmv.restype = ctypes.c_void_p
+    assert not feves_lib.me_create_pmv(*args)
+    assert feves_lib.me_last_error() == -1
+    assert feves_lib.me_set_pmv(None, None) == -1

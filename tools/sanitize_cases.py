@@ -22,4 +22,19 @@ for (W, H, S, n) in [(64, 48, 16, 2), (37, 29, 8, 1), (96, 80, 64, 2), (48, 40, 
         me.stream_push(f)
     torch.cuda.synchronize()
     me.close()
+# G21 predicted-MV centre: predictors at and beyond the clamp, with the rate term (runtime-S ME, SME RD)
+for (W, H, S, n, mp) in [(64, 48, 16, 2, 6), (37, 29, 8, 1, 5), (96, 64, 32, 2, 16)]:
+    frames = [torch.from_numpy(gen_tex(W, H, t, 2)).cuda() for t in range(n + 2)]
+    me = F.MotionEstimator(W, H, S, n, max_pmv=mp)
+    rng = np.random.default_rng(S)
+    pm = torch.from_numpy(rng.integers(-mp - 3, mp + 4, (me.mb_rows * me.mb_cols, n, 2)).astype(np.int16)).cuda()
+    me.set_pmv(pm)
+    me.set_lambda(5)
+    sfs = [me.new_sf() for _ in range(n)]
+    q, qs = me.encode_frame(frames[n], frames[:n], sfs, n_int=n, out_me=me.new_mvs())[1]
+    me.mode_decision(q, qs)
+    for f in frames:
+        me.stream_push(f)
+    torch.cuda.synchronize()
+    me.close()
 print("sanitize cases done")
