@@ -113,6 +113,24 @@ __device__ __forceinline__ uint32_t strip_block_dist(const uint8_t* __restrict__
 // The SF pitch and plane size are multiples of 16 bytes (G11 layout), so a
 // sweep's rows share one alignment: the aligned word pointer and the byte shift
 // are computed once per sweep (RowP) and each row costs 2 LDG + the funnel shifts.
+// SF row word load.  FEVES_SME_L2PF = 128 / 256: the same non-coherent load with an L2
+// sector-promotion hint (experiment knob; 0 = plain __ldg, the default)
+#ifndef FEVES_SME_L2PF
+#define FEVES_SME_L2PF 0
+#endif
+__device__ __forceinline__ uint32_t sf_ld(const uint32_t* p) {
+#if FEVES_SME_L2PF == 128
+  uint32_t v;
+  asm("ld.global.nc.L2::128B.u32 %0, [%1];" : "=r"(v) : "l"(p));
+  return v;
+#elif FEVES_SME_L2PF == 256
+  uint32_t v;
+  asm("ld.global.nc.L2::256B.u32 %0, [%1];" : "=r"(v) : "l"(p));
+  return v;
+#else
+  return __ldg(p);
+#endif
+}
 struct Win2 { uint32_t l, r; };
 struct RowP { const uint32_t* w; uint32_t sh; };
 __device__ __forceinline__ RowP rowp(const uint8_t* p) {
@@ -120,11 +138,11 @@ __device__ __forceinline__ RowP rowp(const uint8_t* p) {
   return {reinterpret_cast<const uint32_t*>(a & ~uintptr_t(3)), 8u * (uint32_t)(a & 3)};
 }
 __device__ __forceinline__ Win2 ld_lr(const RowP& q, int off) {   // off = row * (pitch / 4)
-  const uint32_t w0 = __ldg(q.w + off), w1 = __ldg(q.w + off + 1);
+  const uint32_t w0 = sf_ld(q.w + off), w1 = sf_ld(q.w + off + 1);
   return {__funnelshift_r(w0, w1, q.sh), __funnelshift_rc(w0, w1, q.sh + 8u)};
 }
 __device__ __forceinline__ uint32_t ld_w(const RowP& q, int off) {
-  return __funnelshift_r(__ldg(q.w + off), __ldg(q.w + off + 1), q.sh);
+  return __funnelshift_r(sf_ld(q.w + off), sf_ld(q.w + off + 1), q.sh);
 }
 
 // Half stage, SAD, one block group of HR rows (DESIGN.md §6 "row sweep"): for the
