@@ -51,6 +51,9 @@ def parse():
     ap.add_argument("--pipeline", type=int, default=None, help="ME_OPT_PIPELINE_RF (default: library default)")
     ap.add_argument("--me-ctas", type=int, default=None, help="ME_OPT_ME_CTAS_PER_SM")
     ap.add_argument("--fused", type=int, default=None, help="ME_OPT_FUSED_SME")
+    ap.add_argument("--lam", type=int, default=0, help="f4 variant: rate term lambda (G18); 0 = the paper's SAD")
+    ap.add_argument("--max-pmv", type=int, default=0,
+                    help="f4 variant: predicted-MV centre (G21), predictor = the synthetic motion rounded, clamp K")
     ap.add_argument("--adaptive", action="store_true", help="N>1: re-split MB rows every frame (SURVEY §8 f3)")
     ap.add_argument("--overlap", type=int, default=None,
                     help="ME_OPT_OVERLAP_SME for the e2e stream (SME(t) co-runs with ME(t+1))")
@@ -208,7 +211,8 @@ def config_json(cfg, args):
             "height": cfg.height, "n_rf": cfg.n_rf, "sa_range": cfg.sa_range, "path": "int+me+sme (IPPP stream)",
             "partitions": 41, "parallelism": f"mb-row x{args.gpus}" + (" adaptive" if args.adaptive else "") +
             (f" ({args.exchange} exchange)" if args.gpus > 1 and not args.adaptive else ""),
-            "l2": "flushed (512 MiB write) before every timed step"}
+            "l2": "flushed (512 MiB write) before every timed step",
+            **({"variant": {"lambda": args.lam, "max_pmv": args.max_pmv}} if (args.lam or args.max_pmv) else {})}
 
 
 # --------------------------------------------------------------------- feves --
@@ -246,7 +250,15 @@ def run_feves(args, cfg):
             dist.init_process_group("nccl", device_id=dev)
         else:
             dist.init_process_group(backend)
-    me = feves.MotionEstimator(cfg.width, cfg.height, cfg.sa_range, cfg.n_rf, device=dev)
+    me = feves.MotionEstimator(cfg.width, cfg.height, cfg.sa_range, cfg.n_rf, device=dev, max_pmv=args.max_pmv)
+    if args.lam:
+        me.set_lambda(args.lam)
+    if args.max_pmv:                                 # G21: RF r (frame t-1-r) predicted by the synthetic motion
+        pm = torch.empty((me.mb_rows * me.mb_cols, cfg.n_rf, 2), dtype=torch.int16)
+        for r in range(cfg.n_rf):
+            pm[:, r, 0], pm[:, r, 1] = round(-1.25 * (r + 1)), round(0.75 * (r + 1))
+        pmv_dev = pm.to(dev)
+        me.set_pmv(pmv_dev)
     r0, r1 = stripes(me.mb_rows, world)[rank]
     me.set_rows(r0, r1)      # (ShardedStream may re-split later in adaptive mode)
     for opt, val in ((me.OPT_PIPELINE_RF, args.pipeline), (me.OPT_ME_CTAS_PER_SM, args.me_ctas),

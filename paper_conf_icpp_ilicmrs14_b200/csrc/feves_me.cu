@@ -125,7 +125,10 @@ static cudaError_t set_me_smem(int bytes) {
                   me_fsbm_kernel<0, true>, me_fsbm_kernel<16, true>, me_fsbm_kernel<32, true>,
                   me_fsbm_kernel<64, true>, me_fsbm_kernel<128, true>,
                   me_fsbm_kernel<0, false, 15>, me_fsbm_kernel<16, false, 15>, me_fsbm_kernel<32, false, 15>,
-                  me_fsbm_kernel<64, false, 15>, me_fsbm_kernel<128, false, 15>})
+                  me_fsbm_kernel<64, false, 15>, me_fsbm_kernel<128, false, 15>,
+                  me_fsbm_kernel<16, false, 16, true>, me_fsbm_kernel<32, false, 16, true>,
+                  me_fsbm_kernel<64, false, 16, true>, me_fsbm_kernel<16, false, 15, true>,
+                  me_fsbm_kernel<32, false, 15, true>, me_fsbm_kernel<64, false, 15, true>})
     if (e == cudaSuccess) e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
   return e;
 }
@@ -382,10 +385,12 @@ static int launch_me(me_ctx* c, const uint8_t* cf, const uint8_t* const* rfs, in
 #define FEVES_ME_LAUNCH(SS)                                                              \
   do {                                                                                   \
     if (fused) me_fsbm_kernel<SS, true><<<grid, c->me_threads, smem, st>>>(P);          \
+    else if (c->max_pmv && c->lambda) me_fsbm_kernel<SS, false, 15, true><<<grid, c->me_threads, smem, st>>>(P); \
+    else if (c->max_pmv) me_fsbm_kernel<SS, false, 16, true><<<grid, c->me_threads, smem, st>>>(P); \
     else if (c->lambda) me_fsbm_kernel<SS, false, 15><<<grid, c->me_threads, smem, st>>>(P); \
     else me_fsbm_kernel<SS, false><<<grid, c->me_threads, smem, st>>>(P);               \
   } while (0)
-  switch (c->inclusive || c->max_pmv ? 0 : c->S) {   // compile-time window geometry for the paper's SA sizes (Fig. 6a: 32..256)
+  switch (c->inclusive || (c->max_pmv && c->S == 128) ? 0 : c->S) {   // compile-time window geometry for the paper's SA sizes (Fig. 6a: 32..256)
     case 16: FEVES_ME_LAUNCH(16); break;
     case 32: FEVES_ME_LAUNCH(32); break;
     case 64: FEVES_ME_LAUNCH(64); break;

@@ -357,8 +357,9 @@ __device__ __forceinline__ void fused_sme(const MeParams& P, const uint32_t* cf_
 
 // S_CT = compile-time SA size (0 = any even S read from P at run time);
 // FUSE = also run the SME of this MB (fused_sme) after its ME;
-// KSH = key shift: 16 (pure SAD) or 15 (rate term, G18: J may exceed 16 bits).
-template <int S_CT, bool FUSE = false, int KSH = 16>
+// KSH = key shift: 16 (pure SAD) or 15 (rate term, G18: J may exceed 16 bits);
+// PMV = the G21 predictor is read (always possible in the runtime-S kernel).
+template <int S_CT, bool FUSE = false, int KSH = 16, bool PMV = false>
 // S_CT > 0: <= 128 candidates/axis -> <= 4 warps, 4 CTAs/SM.  S_CT == 0 (runtime S,
 // incl. the inclusive SA's 129 candidates -> 5 warps): same 128-register cap.
 __global__ void __launch_bounds__(S_CT ? 128 : 256, S_CT ? FEVES_ME_MINB : 2) me_fsbm_kernel(const MeParams P) {
@@ -401,10 +402,11 @@ __global__ void __launch_bounds__(S_CT ? 128 : 256, S_CT ? FEVES_ME_MINB : 2) me
 
   for (int ref = 0; ref < P.n_rf; ++ref) {
     const uint8_t* __restrict__ rf = P.rf[ref];
-    // G21: the SA of this (MB, RF) is centred on the clamped predictor p (runtime-S kernel only;
-    // the compile-time kernels never see a predictor, so their code is unchanged)
+    // G21: the SA of this (MB, RF) is centred on the clamped predictor p (runtime-S kernel and the
+    // PMV instantiations; the default compile-time kernels never see a predictor, code unchanged)
+    constexpr bool kPmv = S_CT == 0 || PMV;
     int pcx = 0, pcy = 0;
-    if (S_CT == 0 && P.pmv) {
+    if (kPmv && P.pmv) {
       const size_t pi = ((size_t)mby * P.mb_cols + mbx) * P.rf_stride + ref;
       pcx = min(max((int)P.pmv[2 * pi], -P.max_pmv), P.max_pmv);
       pcy = min(max((int)P.pmv[2 * pi + 1], -P.max_pmv), P.max_pmv);
@@ -447,6 +449,16 @@ __global__ void __launch_bounds__(S_CT ? 128 : 256, S_CT ? FEVES_ME_MINB : 2) me
           const uint4 v = __ldg(reinterpret_cast<const uint4*>(src));
           w[0] = v.x; w[1] = v.y; w[2] = v.z; w[3] = v.w;
           w[4] = __ldg(reinterpret_cast<const uint32_t*>(src + 16));
+        } else if (kPmv && P.vec_ok && x >= 0 && (x & ~3) + 24 <= P.W) {
+          // G21: a predictor moves the window start off the 16-byte grid; the rows are still
+          // aligned, so 6 aligned words + funnel shifts instead of per-byte clamped loads
+          const uint32_t* src = reinterpret_cast<const uint32_t*>(rf + (size_t)y * P.W + (x & ~3));
+          const uint32_t sh = 8u * (uint32_t)(x & 3);
+          uint32_t a[6];
+#pragma unroll
+          for (int i = 0; i < 6; ++i) a[i] = __ldg(src + i);
+#pragma unroll
+          for (int i = 0; i < 5; ++i) w[i] = __funnelshift_r(a[i], a[i + 1], sh);
         } else {
 #pragma unroll
           for (int i = 0; i < 5; ++i) w[i] = load4_clamped(rf, P.W, P.H, x + 4 * i, y);
@@ -566,7 +578,7 @@ __global__ void __launch_bounds__(S_CT ? 128 : 256, S_CT ? FEVES_ME_MINB : 2) me
       uint32_t mv = __ldg(P.inv_tab + rk);                   // SA offset (dx, dy)
       if (KSH != 16)                                         // rate of the offset = R(mv - p) (G21)
         sad -= (uint32_t)(P.lambda * (se_bits(4 * (int)(int16_t)(mv & 0xffffu)) + se_bits(4 * (int)(int16_t)(mv >> 16))));
-      if (S_CT == 0 && P.pmv)                                // mv = p + offset (G21)
+      if (kPmv && P.pmv)                                     // mv = p + offset (G21)
         mv = (uint32_t)(uint16_t)((int)(int16_t)(mv & 0xffffu) + pcx) |
              ((uint32_t)(uint16_t)((int)(int16_t)(mv >> 16) + pcy) << 16);
       const size_t o = ((size_t)(blockIdx.y * P.mb_cols + mbx) * P.rf_stride + ref) * kNPart + p;
