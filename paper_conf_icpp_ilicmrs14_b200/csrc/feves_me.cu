@@ -671,8 +671,8 @@ extern "C" int me_stream_push(me_ctx* c, const uint8_t* cf, int cf_on_host, int1
   // rows of every frame this stripe reads (ME +-R, SME +1, 6-tap -2..+3)
   int y0 = 0, y1 = c->H;
   if (c->halo_only) {
-    y0 = std::max(0, 16 * c->row0 - c->R - 6);
-    y1 = std::min(c->H, 16 * c->row1 + c->R + 7);
+    y0 = std::max(0, 16 * c->row0 - c->R - c->max_pmv - 6);   // + the predictor's reach (G21)
+    y1 = std::min(c->H, 16 * c->row1 + c->R + c->max_pmv + 7);
   }
   const int n_ref = (int)std::min<long long>(t, c->n_rf);
   for (int k = 0; k < n_ref; ++k) {             // a re-split may need rows a halo-only frame lacks

@@ -129,3 +129,35 @@ def test_set_pmv_needs_room(feves):
     with pytest.raises(feves.FevesError):
         me.set_pmv(torch.zeros((12, 1, 2), dtype=torch.int16, device="cuda"))
     me.close()
+
+
+@pytest.mark.parametrize("halo_only", [0, 1])
+def test_pmv_stripes_stream(feves, orc, halo_only):
+    """Predictor on MB-row stripes (the ranks of a sharded run): every stripe's stream push,
+    with only the stripe + (R + max_pmv) halo rows copied when halo_only, == the oracle."""
+    W, H, S, n_rf, max_pmv, lam = 96, 112, 16, 2, 12, 3   # 7 MB rows
+    frames = [gen_tex(W, H, t, 81) for t in range(4)]
+    me = feves.MotionEstimator(W, H, S, n_rf, max_pmv=max_pmv)
+    me.set_lambda(lam)
+    me.set_option(me.OPT_HALO_ONLY, halo_only)
+    n = me.mb_rows * me.mb_cols
+    pm = _field(n, n_rf, 13, max_pmv)
+    pm[:, :, 1] = np.where(np.arange(n)[:, None] % 2 == 0, max_pmv, -max_pmv)   # reach the full halo
+    me.set_pmv(_dev(pm))
+    for r0, r1 in [(0, 3), (3, 5), (5, 7)]:
+        me.set_rows(r0, r1)
+        me.stream_reset()
+        mbs = np.arange(r0 * me.mb_cols, r1 * me.mb_cols, dtype=np.int32)
+        for t, f in enumerate(frames):
+            qm, qs, used = me.stream_push(_dev(f))
+            torch.cuda.synchronize()
+            if used == 0:
+                continue
+            rfs = [frames[t - 1 - k] for k in range(used)]
+            sub = np.ascontiguousarray(pm[:, :used])
+            o_m, _ = orc.me(f, rfs, S, mb_list=mbs, lam=lam, pmv=sub, max_pmv=max_pmv)
+            o_q, o_s = orc.sme(f, rfs, o_m, mb_list=mbs, lam=lam, pmv=sub, max_pmv=max_pmv)
+            k = len(mbs)
+            np.testing.assert_array_equal(qm.cpu().numpy().reshape(k, n_rf, 41, 2)[:, :used], o_q)
+            np.testing.assert_array_equal(qs.cpu().numpy().reshape(k, n_rf, 41)[:, :used], o_s)
+    me.close()
