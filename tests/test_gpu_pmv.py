@@ -161,3 +161,43 @@ def test_pmv_stripes_stream(feves, orc, halo_only):
             np.testing.assert_array_equal(qm.cpu().numpy().reshape(k, n_rf, 41, 2)[:, :used], o_q)
             np.testing.assert_array_equal(qs.cpu().numpy().reshape(k, n_rf, 41)[:, :used], o_s)
     me.close()
+
+
+def test_pmv_full_size_sampled(feves, orc):
+    """BASELINE config[2] size (1080p, 4 RF, S 64) with the rate term and a predictor field
+    (synthetic motion + seeded jitter, some beyond the clamp) through encode_frame, the
+    launch configuration bench.py --lam 4 --max-pmv 8 times; sampled MBs vs the oracle."""
+    from synth import CONFIGS, make_workload
+    from test_gpu_parity import _sample_mbs
+    cfg, lam, max_pmv = CONFIGS["1080p_sa64_4rf"], 4, 8
+    cf, rfs = make_workload(cfg, kind="tex")
+    me = feves.MotionEstimator(cfg.width, cfg.height, cfg.sa_range, cfg.n_rf, max_pmv=max_pmv)
+    me.set_lambda(lam)
+    n = me.mb_rows * me.mb_cols
+    rng = np.random.default_rng(64)
+    pm = rng.integers(-3, 4, (n, cfg.n_rf, 2)).astype(np.int16)
+    for r in range(cfg.n_rf):
+        pm[:, r, 0] += round(-1.25 * (r + 1))
+        pm[:, r, 1] += round(0.75 * (r + 1))
+    pm[::97] = 11                                        # beyond the clamp
+    me.set_pmv(_dev(pm))
+    tcf, trfs = _dev(cf), [_dev(r) for r in rfs]
+    sfs = [me.new_sf() for _ in trfs]
+    (mvs, sads), (qmvs, qsads) = me.encode_frame(tcf, trfs, sfs, n_int=cfg.n_rf, out_me=me.new_mvs())
+    torch.cuda.synchronize()
+    mvs = mvs.cpu().numpy().reshape(n, cfg.n_rf, 41, 2)
+    sads = sads.cpu().numpy().reshape(n, cfg.n_rf, 41)
+    qmvs = qmvs.cpu().numpy().reshape(n, cfg.n_rf, 41, 2)
+    qsads = qsads.cpu().numpy().reshape(n, cfg.n_rf, 41)
+    mbs = np.union1d(_sample_mbs(me.mb_cols, me.mb_rows, 8, 6), np.arange(0, n, 97 * 20, dtype=np.int32))
+    o_m, o_s = orc.me(cf, rfs, cfg.sa_range, mb_list=mbs, lam=lam, pmv=pm, max_pmv=max_pmv)
+    np.testing.assert_array_equal(mvs[mbs], o_m)
+    np.testing.assert_array_equal(sads[mbs], o_s)
+    o_q, o_qs = orc.sme(cf, rfs, o_m, mb_list=mbs, lam=lam, pmv=pm, max_pmv=max_pmv)
+    np.testing.assert_array_equal(qmvs[mbs], o_q)
+    np.testing.assert_array_equal(qsads[mbs], o_qs)
+    # everywhere: every ME MV lies in its clamped predictor's SA
+    p = np.clip(pm, -max_pmv, max_pmv)[:, :, None, :].astype(np.int32)
+    d = mvs.astype(np.int32) - p
+    assert (d >= -cfg.sa_range // 2).all() and (d < cfg.sa_range // 2).all()
+    me.close()
