@@ -47,7 +47,11 @@ def parse():
     ap.add_argument("--e2e-steps", type=int, default=50)
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
-    ap.add_argument("--cpu-budget", type=float, default=10.0, help="seconds of oracle wall time")
+    ap.add_argument("--cpu-budget", type=float, default=10.0,
+                    help="reference arm: seconds of oracle wall time per step (a seeded MB sample)")
+    ap.add_argument("--cpu-frame", choices=["full", "sample"], default="full",
+                    help="cpu_baseline: the oracle on ONE FULL frame on all host cores (default) or a sample")
+    ap.add_argument("--graph", type=int, default=1, help="ME_OPT_GRAPH: one CUDA graph per frame (default 1)")
     ap.add_argument("--pipeline", type=int, default=None, help="ME_OPT_PIPELINE_RF (default: library default)")
     ap.add_argument("--me-ctas", type=int, default=None, help="ME_OPT_ME_CTAS_PER_SM")
     ap.add_argument("--fused", type=int, default=None, help="ME_OPT_FUSED_SME")
@@ -78,10 +82,9 @@ def workload_units(cfg, n_ref=None):
     n_mb = mbc * mbr
     me_cands = n_mb * n_ref * cfg.sa_range ** 2           # MB-candidates (each 256 px-absdiff, 41 SADs)
     sme_px = n_mb * n_ref * 16 * 7 * 256                   # 16 sub-pel candidates x 7 modes x 256 px
-    R = cfg.sa_range // 2
-    pad = -(-(R + 4) // 16) * 16
-    sf_bytes = 16 * (16 * mbr + 2 * pad) * (16 * mbc + 2 * pad)
-    int_bytes = cfg.width * cfg.height + sf_bytes          # read the RF, write 16 planes
+    # INT algorithmic bytes: 1 B read + 15 B written per position of the padded
+    # MB-grid frame (16 B/px; 33.42 MB at 1080p) -- the SF margin rows/columns are not counted
+    int_bytes = 16 * (16 * mbc) * (16 * mbr)
     return dict(n_mb=n_mb, me_cands=me_cands, me_px=me_cands * 256, sme_px=sme_px,
                 gsad=me_cands + sme_px / 256, int_bytes=int_bytes)
 
@@ -133,34 +136,43 @@ class Clocks:
 # ----------------------------------------------------------------- reference --
 
 class OracleSampler:
-    """The oracle (as it stands, never tuned) on a bounded seeded MB sample of one frame."""
+    """The oracle (as it stands, never tuned) on the bench workload: one full frame or a
+    bounded seeded MB sample of it, on a given number of host threads."""
 
-    def __init__(self, cfg):
+    def __init__(self, cfg, threads=None):
         import numpy as np
         import oracle
         from synth import make_workload
 
         oracle.build()
         self.orc, self.cfg = oracle, cfg
-        self.threads = os.cpu_count() or 1
+        self.threads = threads or os.cpu_count() or 1
         self.cf, self.rfs = make_workload(cfg)
         self.n_total = workload_units(cfg)["n_mb"]
         self.order = np.random.default_rng(1234).permutation(self.n_total).astype(np.int32)
         self.layout = oracle.sf_layout(cfg.width, cfg.height, cfg.sa_range)
-        t0 = time.perf_counter()              # calibrate: one MB per thread
+        self.t_cal = None
+
+    def calibrate(self):
+        t0 = time.perf_counter()              # one MB per thread
         self.run(self.threads)
         self.t_cal = time.perf_counter() - t0
 
     def size_for(self, budget_s):
+        if self.t_cal is None:
+            self.calibrate()
         n = self.threads * max(1, round(budget_s / max(self.t_cal, 1e-3)))
         return int(min(self.n_total, n))
 
     def run(self, n):
+        """ME + SME of n MBs (all n_rf RFs) and INT of the matching share of one RF's SF rows.
+        n = n_total is one whole frame (nothing extrapolated)."""
         import numpy as np
         cfg, orc = self.cfg, self.orc
-        mbs = np.sort(self.order[:n])
+        full = n >= self.n_total
+        mbs = None if full else np.sort(self.order[:n])
         pad, pitch, rows = self.layout
-        int_rows = max(1, round(rows * n / self.n_total))
+        int_rows = rows if full else max(1, round(rows * n / self.n_total))
         t0 = time.perf_counter()
         mv, _ = orc.me(self.cf, self.rfs, cfg.sa_range, mb_list=mbs, threads=self.threads)
         t1 = time.perf_counter()
@@ -169,36 +181,55 @@ class OracleSampler:
         orc.int_planes(self.rfs[0], pad, pitch, rows, row_begin=0, row_end=int_rows, threads=self.threads)
         t3 = time.perf_counter()
         t = t3 - t0
-        fps = (n / self.n_total) / t
+        fps = (min(n, self.n_total) / self.n_total) / t
+        what = (f"one FULL frame: {self.n_total} MBs x {cfg.n_rf} RFs ME+SME and all {rows} SF rows of one INT "
+                f"(the newest RF; stream mode)" if full else
+                f"{n} of {self.n_total} MBs (seeded) x {cfg.n_rf} RFs ME+SME and {int_rows} of {rows} SF rows of "
+                f"one INT, extrapolated linearly (FSBM work is linear in MBs, P:260)")
         return {"value": fps, "unit": "frames/s", "cores": self.threads, "kind": "oracle",
-                "sample": f"{n} of {self.n_total} MBs (seeded) x {cfg.n_rf} RFs ME+SME and {int_rows} of {rows} "
-                          f"SF rows of one INT ({t:.1f} s wall on {self.threads} threads), extrapolated linearly "
-                          f"(FSBM work is linear in MBs, P:260)",
-                "seconds": {"me": t1 - t0, "sme": t2 - t1, "int": t3 - t2},
+                "sample": f"{what}; {t:.1f} s wall on {self.threads} thread(s)",
+                "seconds": {"me": t1 - t0, "sme": t2 - t1, "int": t3 - t2, "total": t},
+                "extrapolated": not full,
                 "candidate_gsad_per_s": workload_units(cfg)["gsad"] * fps / 1e9}
 
 
-def cpu_oracle_sample(cfg, budget_s):
+def cpu_baseline(cfg, args):
+    """cpu_baseline of the bench line: the oracle on one full frame on all host cores
+    (measured, not extrapolated), plus a single-thread timing on one MB row of it."""
     s = OracleSampler(cfg)
-    return s.run(s.size_for(budget_s))
+    cb = s.run(s.n_total if args.cpu_frame == "full" else s.size_for(args.cpu_budget))
+    one = OracleSampler(cfg, threads=1)
+    mbc = -(-cfg.width // 16)
+    st = one.run(mbc)                       # a seeded sample of one MB row's worth of MBs
+    cb["single_thread"] = {"value": st["value"], "unit": "frames/s", "cores": 1, "sample": st["sample"],
+                           "speedup_all_cores": cb["value"] / st["value"]}
+    return cb
 
 
 def run_reference(args, cfg):
+    """--impl reference: the oracle as it stands, on all host cores, each step a bounded seeded
+    MB sample of the bench workload (about --cpu-budget s, capped so the whole warm-up + timed run
+    takes ~150 s).  ms_per_step is the MEASURED wall time of one such step; value is that step's
+    frames/s (sample share / wall time) -- extrapolated from the sample, as its cpu_baseline says."""
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
         return
     s = OracleSampler(cfg)
     n = s.size_for(min(args.cpu_budget, 150.0 / (args.steps + args.warmup)))
-    vals, cb = [], None
+    walls, cb = [], None
     for i in range(args.warmup + args.steps):
+        t0 = time.perf_counter()
         cb = s.run(n)
         if i >= args.warmup:
-            vals.append(cb["value"])
-    v = statistics.mean(vals)
+            walls.append(time.perf_counter() - t0)
+    step_s = statistics.mean(walls)
+    v = (n / s.n_total) / step_s
     line = {"impl": "reference", "metric": METRIC, "value": v, "unit": "frames/s", "n_gpus": args.gpus,
-            "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 / v, "higher_is_better": True,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": step_s * 1e3, "higher_is_better": True,
             "scaling": "strong", "vs_baseline": None, "dtype": "u8",
             "data": "synthetic (gen-tex, seeded)", "config": config_json(cfg, args),
+            "step": f"one step = the oracle on a seeded sample of {n} of {s.n_total} MBs of the frame "
+                    f"({100.0 * n / s.n_total:.1f}%), all {cfg.n_rf} RFs, ME+SME+INT share",
             "cpu_baseline": {"kind": cb["kind"], "cores": cb["cores"], "sample": cb["sample"], "value": v,
                              "unit": "frames/s"},
             "e2e": {"value": v, "unit": "frames/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
@@ -212,6 +243,8 @@ def config_json(cfg, args):
             "partitions": 41, "parallelism": f"mb-row x{args.gpus}" + (" adaptive" if args.adaptive else "") +
             (f" ({args.exchange} exchange)" if args.gpus > 1 and not args.adaptive else ""),
             "l2": "flushed (512 MiB write) before every timed step",
+            "graph": "one CUDA graph per frame (ME_OPT_GRAPH)" if args.impl == "feves" and args.graph and args.gpus == 1
+            else "none",
             **({"variant": {"lambda": args.lam, "max_pmv": args.max_pmv}} if (args.lam or args.max_pmv) else {})}
 
 
@@ -262,7 +295,7 @@ def run_feves(args, cfg):
     r0, r1 = stripes(me.mb_rows, world)[rank]
     me.set_rows(r0, r1)      # (ShardedStream may re-split later in adaptive mode)
     for opt, val in ((me.OPT_PIPELINE_RF, args.pipeline), (me.OPT_ME_CTAS_PER_SM, args.me_ctas),
-                     (me.OPT_FUSED_SME, args.fused)):
+                     (me.OPT_FUSED_SME, args.fused), (me.OPT_GRAPH, args.graph if world == 1 else None)):
         if val is not None:
             me.set_option(opt, val)
     me.set_timing(True)
@@ -347,6 +380,21 @@ def run_feves(args, cfg):
         iso_r.append((a, b))
     torch.cuda.synchronize()
     int_iso_clean_ms = statistics.mean(a.elapsed_time(b) for a, b in iso_r)
+    # "stateless" INT: all n_rf RFs of a frame interpolated back to back, as
+    # me_encode_frame(n_int = n_rf) does without the stream's SF ring, L2 flushed before
+    sfs_all = [sf_scratch] + [me.new_sf() for _ in range(cfg.n_rf - 1)]
+    iso_s = []
+    for k in range(max(5, min(args.steps, 20))):
+        flush.max()
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record(stream)
+        for r in range(cfg.n_rf):
+            me.interpolate(frames[(k + r) % n_frames], out=sfs_all[r])
+        b.record(stream)
+        iso_s.append((a, b))
+    torch.cuda.synchronize()
+    int_stateless_ms = statistics.mean(a.elapsed_time(b) for a, b in iso_s)
+    del sfs_all
     del sf_scratch
     me.set_timing(True)
 
@@ -430,6 +478,7 @@ def run_feves(args, cfg):
         e0.record(stream)
         for i in range(args.e2e_steps):
             me.stream_push(pinned[(cfg.n_rf + 2 + i) % n_frames], out=(qm_h, qs_h))
+        me.stream_join()                     # the last frame's D2H (copy-out stream) is inside the region
         e1.record(stream)
         me.sync()
         torch.cuda.synchronize()
@@ -446,7 +495,7 @@ def run_feves(args, cfg):
         return
     cpu = None
     if not args.no_cpu_baseline and world == 1:
-        cpu = cpu_oracle_sample(cfg, args.cpu_budget)
+        cpu = cpu_baseline(cfg, args)
     line = {
         "metric": METRIC, "value": fps, "unit": "frames/s", "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": total_ms / args.steps, "higher_is_better": True,
@@ -457,6 +506,7 @@ def run_feves(args, cfg):
         "px_absdiff_per_s": (u["me_px"] + u["sme_px"]) * fps,
         "kernels_ms": {"int": int_ms, ("me_sme_fused" if fused else "me"): me_ms, "sme": sme_ms,
                        "int_isolated": int_iso_ms, "int_isolated_clean_l2": int_iso_clean_ms,
+                       "int_stateless_all_rf": int_stateless_ms,
                        "me_only_isolated": me_only_ms,
                        "note": "CUDA events around each launch on its own stream" + (
                            "; fused: INT(t-1) then one ME+SME kernel" if fused else
@@ -477,6 +527,12 @@ def run_feves(args, cfg):
                              "achieved": me_only_px / 1e12, "peak": peak_px / 1e12, "unit": "Tpx-absdiff/s",
                              "frac": me_only_px / peak_px},
         "roofline_int": {"bound": "hbm", "kernel": "int_subpel_kernel",
+                         "traffic_unit": "16 B per position of the padded MB-grid frame (SURVEY §8(d): 1 B read "
+                                         "+ 15 B written)",
+                         "limiter": "issue / latency, not HBM (ncu: the planes land in L2; DESIGN.md §6)",
+                         "stateless_all_rf": {"ms": int_stateless_ms, "frames_rf": cfg.n_rf,
+                                              "achieved_gbs": cfg.n_rf * u["int_bytes"] * stripe_frac /
+                                              (int_stateless_ms / 1e3) / 1e9},
                          "timing": "isolated, L2 flushed by a 512 MiB read (cold, clean lines); after a 512 MiB "
                                    "write flush (dirty lines to write back) see kernels_ms.int_isolated",
                          "achieved": u["int_bytes"] * stripe_frac / (int_iso_clean_ms / 1e3) / 1e9,

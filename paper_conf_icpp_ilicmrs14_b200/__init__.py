@@ -58,18 +58,19 @@ def lib():
         L.me_stream_reset.argtypes = [P]
         L.me_stream_push.argtypes = [P, P, i, P, P, i, P]
         L.me_stream_outputs.argtypes = [P, P, P]
+        L.me_stream_join.argtypes = [P]
         L.me_sync.argtypes = [P]
         L.me_set_timing.argtypes = [P, i]
         L.me_get_timings.argtypes = [P, P, P, P]
         L.me_set_fused.argtypes = [P, i]
         L.me_set_option.argtypes = [P, i, i]
-        L.me_mode_decision.argtypes = [P, P, P, P]
+        L.me_mode_decision.argtypes = [P, P, P, i, P]
         L.me_ipc_export.argtypes = [P, P, P, ctypes.POINTER(ctypes.c_size_t)]
         L.me_ipc_open.argtypes = [P, P, ctypes.c_size_t, ctypes.c_size_t, ctypes.POINTER(ctypes.c_void_p)]
         L.me_ipc_close.argtypes = [P, P]
         for fn in ("me_set_stream", "me_set_rows", "me_get_layout", "me_estimate", "int_interpolate",
                    "sme_refine", "me_encode_frame", "me_last_launch_count", "me_stream_reset",
-                   "me_stream_push", "me_stream_outputs", "me_sync", "me_set_timing", "me_get_timings", "me_set_fused", "me_set_option", "me_mode_decision",
+                   "me_stream_push", "me_stream_outputs", "me_stream_join", "me_sync", "me_set_timing", "me_get_timings", "me_set_fused", "me_set_option", "me_mode_decision",
                    "me_ipc_export", "me_ipc_open", "me_ipc_close"):
             getattr(L, fn).restype = i
         _lib = L
@@ -85,6 +86,29 @@ def _dev_u8(t, name):
     if not (isinstance(t, torch.Tensor) and t.is_cuda and t.dtype == torch.uint8 and t.is_contiguous()):
         raise FevesError(f"{name}: expected a contiguous uint8 CUDA tensor")
     return t
+
+
+def _check_out(mv_shape, mvs, sads, name, device=None, host_ok=False):
+    """out= buffers: the C-ABI cannot check sizes, so a wrong-size or wrong-kind buffer
+    would become an out-of-bounds device (or, via the async D2H, host) write."""
+    n = 1
+    for d in mv_shape:
+        n *= d
+    for t, dt, k in ((mvs, (torch.int16,), 2), (sads, (torch.uint16, torch.int16), 1)):
+        if t is None:
+            continue
+        if not isinstance(t, torch.Tensor) or t.dtype not in dt or not t.is_contiguous() or t.numel() != n * k:
+            raise FevesError(f"{name}: expected contiguous {dt[0]} tensors with {n * k} elements "
+                             f"(shape {tuple(mv_shape) + ((2,) if k == 2 else ())})")
+        if t.is_cuda:
+            if device is not None and t.device != device:
+                raise FevesError(f"{name}: tensor on {t.device}, context on {device}")
+        elif not host_ok:
+            raise FevesError(f"{name}: expected CUDA tensors")
+        elif not t.is_pinned():
+            raise FevesError(f"{name}: host outputs must be pinned (they are written by an async copy)")
+    if sads is not None and mvs.is_cuda != sads.is_cuda:
+        raise FevesError(f"{name}: both outputs on the device or both on the host")
 
 
 def _ptrs(ts):
@@ -161,6 +185,7 @@ class MotionEstimator:
         for r in rfs:
             _dev_u8(r, "rf")
         mvs, sads = out if out is not None else self.new_mvs()
+        _check_out(self.mv_shape(), mvs, sads, "estimate(out=)", self.device)
         self._bind_stream()
         _check(lib().me_estimate(self._ctx, cf.data_ptr(), _ptrs(rfs), mvs.data_ptr(), sads.data_ptr()))
         return mvs, sads
@@ -169,6 +194,9 @@ class MotionEstimator:
         """INT (int_interpolate): 16 phase planes [16, sf_rows, sf_pitch] u8."""
         _dev_u8(rf, "rf")
         sf = self.new_sf() if out is None else out
+        _dev_u8(sf, "interpolate(out=)")
+        if sf.numel() != N_PHASE * self.sf_rows * self.sf_pitch:
+            raise FevesError(f"interpolate(out=): need {self.sf_shape()} bytes")
         self._bind_stream()
         _check(lib().int_interpolate(self._ctx, rf.data_ptr(), sf.data_ptr()))
         return sf
@@ -178,6 +206,8 @@ class MotionEstimator:
         _dev_u8(cf, "cf")
         assert len(sfs) == self.n_rf
         qmvs, qsads = out if out is not None else self.new_mvs()
+        _check_out(self.mv_shape(), qmvs, qsads, "refine(out=)", self.device)
+        _check_out(self.mv_shape(), mvs, sads, "refine(mvs, sads)", self.device)
         self._bind_stream()
         _check(lib().sme_refine(self._ctx, cf.data_ptr(), _ptrs(sfs), mvs.data_ptr(),
                                 None if sads is None else sads.data_ptr(), qmvs.data_ptr(), qsads.data_ptr()))
@@ -187,6 +217,9 @@ class MotionEstimator:
         """INT (first n_int RFs) -> ME -> SME in one C call (me_encode_frame)."""
         qmvs, qsads = out_sme if out_sme is not None else self.new_mvs()
         mvs, sads = out_me if out_me is not None else (None, None)
+        _check_out(self.mv_shape(), qmvs, qsads, "encode_frame(out_sme=)", self.device)
+        if out_me is not None:
+            _check_out(self.mv_shape(), mvs, sads, "encode_frame(out_me=)", self.device)
         self._bind_stream()
         _check(lib().me_encode_frame(self._ctx, cf.data_ptr(), _ptrs(rfs), _ptrs(sfs), n_int,
                                      None if mvs is None else mvs.data_ptr(),
@@ -206,6 +239,7 @@ class MotionEstimator:
             raise FevesError("cf: expected a contiguous uint8 tensor")
         on_host = not cf.is_cuda
         qmvs, qsads = out if out is not None else self.new_mvs()
+        _check_out(self.mv_shape(), qmvs, qsads, "stream_push(out=)", self.device, host_ok=True)
         out_host = not qmvs.is_cuda
         n = ctypes.c_int()
         if bind_stream:
@@ -226,6 +260,12 @@ class MotionEstimator:
 
     def sync(self):
         _check(lib().me_sync(self._ctx))
+
+    def stream_join(self):
+        """The context (= torch current) stream waits for the internal copy / side streams
+        (me_stream_join): an event recorded after this marks the end of every push so far."""
+        self._bind_stream()
+        _check(lib().me_stream_join(self._ctx))
 
     # ------------------------------------------------- peer memory (8e) --
     def ipc_export(self, t):
@@ -251,7 +291,7 @@ class MotionEstimator:
         _check(lib().me_set_fused(self._ctx, int(on)))
 
     OPT_FUSED_SME, OPT_PIPELINE_RF, OPT_ME_CTAS_PER_SM, OPT_LAMBDA, OPT_SME_SATD, OPT_SA_INCLUSIVE = 1, 2, 3, 4, 5, 6
-    OPT_HALO_ONLY, OPT_OVERLAP_SME = 7, 8
+    OPT_HALO_ONLY, OPT_OVERLAP_SME, OPT_GRAPH = 7, 8, 9
 
     def set_sa_inclusive(self, on: bool = True):
         """Candidates in [-S/2, +S/2]^2 (G1 alternative reading, f4)."""
@@ -276,13 +316,18 @@ class MotionEstimator:
         _check(lib().me_set_pmv(self._ctx, None if pmv is None else pmv.data_ptr()))
         self._pmv = pmv
 
-    def mode_decision(self, qmvs, qsads, out=None):
-        """Best H.264 P-MB configuration per MB (f2, me_mode_decision):
+    def mode_decision(self, qmvs, qsads, out=None, n_ref=None):
+        """Best H.264 P-MB configuration per MB (f2, me_mode_decision) over RF slots
+        [0, n_ref) (default n_rf; pass stream_push's n_ref_used on the first frames):
         int32 [rows, mb_cols, 10] = mb_type, sub_type x4, ref per 8x8 x4, cost."""
-        o = out if out is not None else torch.empty((self.row1 - self.row0, self.mb_cols, 10), dtype=torch.int32,
-                                                    device=self.device)
+        _check_out(self.mv_shape(), qmvs, qsads, "mode_decision(qmvs, qsads)", self.device)
+        shape = (self.row1 - self.row0, self.mb_cols, 10)
+        o = out if out is not None else torch.empty(shape, dtype=torch.int32, device=self.device)
+        if o.dtype != torch.int32 or not o.is_cuda or not o.is_contiguous() or o.numel() != shape[0] * shape[1] * 10:
+            raise FevesError(f"mode_decision(out=): need a contiguous int32 CUDA tensor {shape}")
         self._bind_stream()
-        _check(lib().me_mode_decision(self._ctx, qmvs.data_ptr(), qsads.data_ptr(), o.data_ptr()))
+        _check(lib().me_mode_decision(self._ctx, qmvs.data_ptr(), qsads.data_ptr(),
+                                      self.n_rf if n_ref is None else int(n_ref), o.data_ptr()))
         return o
 
     def set_option(self, option: int, value: int):

@@ -16,9 +16,8 @@
 #include <vector>
 
 #include "int_subpel.cuh"
-#include "me_fsbm.cuh"
+#include "launch.cuh"   // ME / SME launches (their own translation units: me_s*.cu, sme.cu)
 #include "mode_decision.cuh"
-#include "sme_refine.cuh"
 
 using namespace feves;
 
@@ -28,7 +27,7 @@ struct me_ctx {
   int sf_pad, sf_pitch, sf_rows;
   int device;
   cudaStream_t stream;
-  bool own_stream;
+  cudaStream_t own;      // the context's own stream (created in me_create, destroyed in me_destroy)
   uint32_t* d_rank;      // [S][Sp]: [dx+R][dy+R], column pitch Sp = S rounded up to 4 (me_rank_pitch)
   uint32_t* d_inv;       // [(S+1)^2]
   uint32_t* d_glob;      // [4][4096]: S = 128 quadrant-local rank -> global dense rank
@@ -38,8 +37,6 @@ struct me_ctx {
   int me_threads;
   size_t me_smem;
   int last_launches;
-  const void* checked[64];
-  int n_checked;
   // IPPP stream state (me_stream_push): ring of n_rf+1 frames, n_rf SFs
   uint8_t* ring;         // (n_rf+1) * W*H
   uint8_t* sf_ring;      // n_rf * 16*sf_rows*sf_pitch
@@ -84,6 +81,21 @@ struct me_ctx {
   int fv0[kMaxRf + 2], fv1[kMaxRf + 2];   // frame rows each frame-ring slot holds
   struct Peer { uintptr_t lo, hi; void* base; } peers[16];   // me_ipc_open mappings
   int n_peers;
+  cudaEvent_t ev_switch;   // me_set_stream: orders the old stream's work before the new one's
+  // ME_OPT_GRAPH: one captured CUDA graph per ring phase of the device-resident stream
+  struct Graph {
+    cudaGraphExec_t exec;
+    cudaGraph_t graph;     // kept: its frame-copy node is re-pointed at each replay's frame
+    cudaGraphNode_t copy;  // the frame's D2D copy into the ring slot
+    const void* cf; const void* qm; const void* qs;
+    int row0, row1;
+    long long epoch;
+    int timing, launches, timed_mask;
+  };
+  std::vector<Graph> graphs;
+  int graph;             // ME_OPT_GRAPH
+  bool capturing;        // push_enqueue runs inside a stream capture
+  long long gepoch;      // bumped by every setting change: cached graphs are stale
 };
 
 static thread_local int g_last_error = ME_OK;
@@ -106,31 +118,30 @@ static bool is_peer_ptr(const me_ctx* c, const void* p) {
   return false;
 }
 
+// checked on every call (no cache: a freed and re-allocated range must be re-checked)
 static bool is_device_ptr(me_ctx* c, const void* p) {
   if (!p) return false;
   if (is_peer_ptr(c, p)) return true;   // peer memory mapped by me_ipc_open (another GPU's buffer)
-  for (int i = 0; i < c->n_checked; ++i)
-    if (c->checked[i] == p) return true;
   cudaPointerAttributes a;
   if (cudaPointerGetAttributes(&a, p) != cudaSuccess) { cudaGetLastError(); return false; }
-  if (!(a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged) || a.device != c->device) return false;
-  c->checked[c->n_checked % 64] = p;
-  if (c->n_checked < 64) c->n_checked++;
-  return true;
+  return (a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged) && a.device == c->device;
 }
 
 static cudaError_t set_me_smem(int bytes) {
-  cudaError_t e = cudaSuccess;
-  for (auto fn : {me_fsbm_kernel<0>, me_fsbm_kernel<16>, me_fsbm_kernel<32>, me_fsbm_kernel<64>, me_fsbm_kernel<128>,
-                  me_fsbm_kernel<0, true>, me_fsbm_kernel<16, true>, me_fsbm_kernel<32, true>,
-                  me_fsbm_kernel<64, true>, me_fsbm_kernel<128, true>,
-                  me_fsbm_kernel<0, false, 15>, me_fsbm_kernel<16, false, 15>, me_fsbm_kernel<32, false, 15>,
-                  me_fsbm_kernel<64, false, 15>, me_fsbm_kernel<128, false, 15>,
-                  me_fsbm_kernel<16, false, 16, true>, me_fsbm_kernel<32, false, 16, true>,
-                  me_fsbm_kernel<64, false, 16, true>, me_fsbm_kernel<16, false, 15, true>,
-                  me_fsbm_kernel<32, false, 15, true>, me_fsbm_kernel<64, false, 15, true>})
-    if (e == cudaSuccess) e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
+  cudaError_t e = me_set_smem_0(bytes);
+  if (e == cudaSuccess) e = me_set_smem_16(bytes);
+  if (e == cudaSuccess) e = me_set_smem_32(bytes);
+  if (e == cudaSuccess) e = me_set_smem_64(bytes);
+  if (e == cudaSuccess) e = me_set_smem_128(bytes);
   return e;
+}
+
+static void graphs_drop(me_ctx* c) {
+  for (auto& g : c->graphs) {
+    if (g.exec) cudaGraphExecDestroy(g.exec);
+    if (g.graph) cudaGraphDestroy(g.graph);
+  }
+  c->graphs.clear();
 }
 
 static int launch_status() {
@@ -142,7 +153,16 @@ static int launch_status() {
 // key addend table E[dy+R][dx+R] = lambda * R(4dx, 4dy) * kmul + spiral rank (G4, G18):
 // with lambda = 0 this is the spiral rank and key = SAD * 2^16 + rank; with a rate
 // term J = SAD + lambda*R may exceed 16 bits, so key = J * 2^15 + rank (rank < 2^15
-// for S <= 128, J < 2^17 for lambda <= 2000).
+// for S <= 128).  The key is 32 bits, so J must stay below 2^17: with the 16x16 SAD
+// up to 65280 that caps lambda at (2^17 - 1 - 65280) / max R over the SA offsets
+// (lambda_limit: 1935 at S = 64, 1731 at S = 128; the API's own cap is 2000).
+static int lambda_limit(int S, int inclusive) {
+  const int R = S / 2, hi = S + inclusive - 1 - R;
+  int rmax = 0;
+  for (int d = -R; d <= hi; ++d) rmax = std::max(rmax, se_bits(4 * d));
+  return std::min(2000, ((1 << 17) - 1 - 65280) / (2 * rmax));
+}
+
 // Host-only construction of the three ME key tables (no CUDA call; me_key_tables exposes it).
 // e: [Sc][Sp] key addends, [dx+R][dy+R]; inv: dense rank -> packed MV; glob: S = 128 quadrant map.
 static void build_key_tables(int S, int inclusive, int lambda, std::vector<uint32_t>& e, std::vector<uint32_t>& inv,
@@ -182,7 +202,7 @@ static void build_key_tables(int S, int inclusive, int lambda, std::vector<uint3
 extern "C" int me_key_tables(int sa_range, int inclusive, int lambda, uint32_t* key_addend, uint32_t* inv,
                              uint32_t* glob) {
   if (sa_range < 4 || sa_range > 128 || (sa_range & 1) || (inclusive != 0 && inclusive != 1) || lambda < 0 ||
-      lambda > 2000 || !key_addend || !inv || !glob)
+      lambda > lambda_limit(sa_range, inclusive) || !key_addend || !inv || !glob)
     return ME_EINVAL;
   std::vector<uint32_t> e, iv, g;
   build_key_tables(sa_range, inclusive, lambda, e, iv, g);
@@ -246,9 +266,9 @@ extern "C" me_ctx* me_create_pmv(int width, int height, int sa_range, int n_rf, 
             cudaMalloc(&c->d_glob, (size_t)4 * 4096 * 4) == cudaSuccess &&
             cudaMalloc(&c->d_mvs, nmv * 4) == cudaSuccess &&
             cudaMalloc(&c->d_sads, nmv * 2) == cudaSuccess &&
-            cudaStreamCreateWithFlags(&c->stream, cudaStreamNonBlocking) == cudaSuccess;
+            cudaStreamCreateWithFlags(&c->own, cudaStreamNonBlocking) == cudaSuccess;
   if (ok) {
-    c->own_stream = true;
+    c->stream = c->own;
     ok = upload_key_table(c) == ME_OK &&
          set_me_smem(200 * 1024) == cudaSuccess;   // max; the launch asks for what it needs
   }
@@ -265,6 +285,7 @@ extern "C" me_ctx* me_create_pmv(int width, int height, int sa_range, int n_rf, 
 extern "C" void me_destroy(me_ctx* c) {
   if (!c) return;
   if (c->stream) cudaStreamSynchronize(c->stream);
+  if (c->own) cudaStreamSynchronize(c->own);
   if (c->copy_in) cudaStreamSynchronize(c->copy_in);
   if (c->copy_out) cudaStreamSynchronize(c->copy_out);
   if (c->side) cudaStreamSynchronize(c->side);
@@ -296,7 +317,9 @@ extern "C" void me_destroy(me_ctx* c) {
   if (c->side) cudaStreamDestroy(c->side);
   if (c->ev_fork) cudaEventDestroy(c->ev_fork);
   if (c->ev_join) cudaEventDestroy(c->ev_join);
-  if (c->own_stream && c->stream) cudaStreamDestroy(c->stream);
+  if (c->ev_switch) cudaEventDestroy(c->ev_switch);
+  graphs_drop(c);
+  if (c->own) cudaStreamDestroy(c->own);
   for (int i = 0; i < c->n_peers; ++i)
     if (c->peers[i].base) cudaIpcCloseMemHandle(c->peers[i].base);
   if (c->ov_st) { cudaStreamSynchronize(c->ov_st); cudaStreamDestroy(c->ov_st); }
@@ -319,17 +342,26 @@ extern "C" const char* me_strerror(int s) {
   }
 }
 
+// ME_STREAM_OWN = the context's own stream again (it lives until me_destroy).  Work
+// already enqueued on the previous stream is ordered before later work by an event
+// (no host synchronisation).
 extern "C" int me_set_stream(me_ctx* c, void* s) {
   if (!c) return ME_EINVAL;
-  if (c->own_stream && c->stream) { cudaStreamSynchronize(c->stream); cudaStreamDestroy(c->stream); }
-  c->own_stream = false;
-  c->stream = (cudaStream_t)s;
+  cudaStream_t ns = s == ME_STREAM_OWN ? c->own : (cudaStream_t)s;
+  if (ns == c->stream) return ME_OK;
+  if (!c->ev_switch && cudaEventCreateWithFlags(&c->ev_switch, cudaEventDisableTiming) != cudaSuccess)
+    return launch_status();
+  if (cudaEventRecord(c->ev_switch, c->stream) != cudaSuccess || cudaStreamWaitEvent(ns, c->ev_switch, 0) != cudaSuccess)
+    return launch_status();
+  c->stream = ns;
+  c->gepoch++;
   return ME_OK;
 }
 
 extern "C" int me_set_rows(me_ctx* c, int r0, int r1) {
   if (!c || r0 < 0 || r1 > c->mb_rows || r0 >= r1) return ME_EINVAL;
   c->row0 = r0; c->row1 = r1;
+  c->gepoch++;
   return ME_OK;
 }
 
@@ -348,7 +380,10 @@ extern "C" int me_last_launch_count(const me_ctx* c) { return c ? c->last_launch
 
 // --------------------------------------------------------------- launches ----
 static void tmark(me_ctx* c, int i, cudaStream_t st) {
-  if (c->timing) { cudaEventRecord(c->ev_t[i], st); c->timed_mask |= 1 << (i / 2); }
+  if (!c->timing) return;
+  if (c->capturing) cudaEventRecordWithFlags(c->ev_t[i], st, cudaEventRecordExternal);   // a graph node
+  else cudaEventRecord(c->ev_t[i], st);
+  c->timed_mask |= 1 << (i / 2);
 }
 
 // ME (and, when sfs != NULL, the fused SME of me_fsbm.cuh) over n_ref RFs
@@ -382,22 +417,18 @@ static int launch_me(me_ctx* c, const uint8_t* cf, const uint8_t* const* rfs, in
   if (c->me_ctas_per_sm > 0)   // occupancy cap: leave registers / warps for a co-running SME
     smem = std::max(smem, (size_t)(228 * 1024) / (size_t)(c->me_ctas_per_sm + 1) - 1024 + 64);
   tmark(c, 2, st);
-#define FEVES_ME_LAUNCH(SS)                                                              \
-  do {                                                                                   \
-    if (fused) me_fsbm_kernel<SS, true><<<grid, c->me_threads, smem, st>>>(P);          \
-    else if (c->max_pmv && c->lambda) me_fsbm_kernel<SS, false, 15, true><<<grid, c->me_threads, smem, st>>>(P); \
-    else if (c->max_pmv) me_fsbm_kernel<SS, false, 16, true><<<grid, c->me_threads, smem, st>>>(P); \
-    else if (c->lambda) me_fsbm_kernel<SS, false, 15><<<grid, c->me_threads, smem, st>>>(P); \
-    else me_fsbm_kernel<SS, false><<<grid, c->me_threads, smem, st>>>(P);               \
-  } while (0)
+  const int variant = fused ? kMeFused
+                    : c->max_pmv ? (c->lambda ? kMePmvRate : kMePmv)
+                    : c->lambda ? kMeRate : kMePlain;
+  cudaError_t e;
   switch (c->inclusive || (c->max_pmv && c->S == 128) ? 0 : c->S) {   // compile-time window geometry for the paper's SA sizes (Fig. 6a: 32..256)
-    case 16: FEVES_ME_LAUNCH(16); break;
-    case 32: FEVES_ME_LAUNCH(32); break;
-    case 64: FEVES_ME_LAUNCH(64); break;
-    case 128: FEVES_ME_LAUNCH(128); break;
-    default: FEVES_ME_LAUNCH(0); break;
+    case 16: e = me_launch_16(variant, grid, c->me_threads, smem, st, P); break;
+    case 32: e = me_launch_32(variant, grid, c->me_threads, smem, st, P); break;
+    case 64: e = me_launch_64(variant, grid, c->me_threads, smem, st, P); break;
+    case 128: e = me_launch_128(variant, grid, c->me_threads, smem, st, P); break;
+    default: e = me_launch_0(variant, grid, c->me_threads, smem, st, P); break;
   }
-#undef FEVES_ME_LAUNCH
+  if (e != cudaSuccess) { fprintf(stderr, "feves_me: ME launch: %s\n", cudaGetErrorString(e)); return ME_ECUDA; }
   tmark(c, 3, st);
   c->last_launches++;
   return launch_status();
@@ -429,7 +460,8 @@ static int launch_int(me_ctx* c, const uint8_t* rf, uint8_t* sf, cudaStream_t st
   P.border_bx = bx;
   const int nrows = P.row_end - P.row_begin;
   const dim3 block(32, 4);
-  const dim3 grid(std::max(1, (g_hi - g_lo + 31) / 32), (nrows + 3) / 4, nb > 0 ? 2 : 1);
+  // x: interior blocks of 32 groups, or the border slices of bx groups (z = 0), whichever is more
+  const dim3 grid(std::max(std::max(1, (g_hi - g_lo + 31) / 32), (nb + bx - 1) / bx), (nrows + 3) / 4, nb > 0 ? 2 : 1);
   tmark(c, 0, st);
   int_subpel_kernel<<<grid, block, 0, st>>>(P);
   c->last_launches++;
@@ -457,17 +489,13 @@ static int launch_sme(me_ctx* c, const uint8_t* cf, const uint8_t* const* sfs, c
   P.pad = c->sf_pad; P.pitch = c->sf_pitch;
   P.plane = (size_t)c->sf_rows * c->sf_pitch;
   P.fence = is_peer_ptr(c, out_qmvs) || is_peer_ptr(c, out_sads);
+  P.cf_vec = (c->W % 4 == 0) && ((reinterpret_cast<uintptr_t>(cf) & 3) == 0);   // aligned CF word loads
   P.k_hi = kAvgHi;
   const int warps = n_ref * P.n_rows * P.groups;
   tmark(c, 4, st);
   const dim3 sg((warps + 3) / 4, 7);   // y = partition mode
-  if (c->satd) {
-    if (c->lambda) sme_refine_kernel<true, true><<<sg, 128, 0, st>>>(P);
-    else sme_refine_kernel<false, true><<<sg, 128, 0, st>>>(P);
-  } else {
-    if (c->lambda) sme_refine_kernel<true, false><<<sg, 128, 0, st>>>(P);
-    else sme_refine_kernel<false, false><<<sg, 128, 0, st>>>(P);
-  }
+  const cudaError_t e = sme_launch(c->lambda != 0, c->satd != 0, sg, 128, st, P);
+  if (e != cudaSuccess) { fprintf(stderr, "feves_me: SME launch: %s\n", cudaGetErrorString(e)); return ME_ECUDA; }
   tmark(c, 5, st);
   c->last_launches++;
   return launch_status();
@@ -580,6 +608,7 @@ extern "C" int me_encode_frame(me_ctx* c, const uint8_t* cf, const uint8_t* cons
 extern "C" int me_stream_reset(me_ctx* c) {
   if (!c) return ME_EINVAL;
   c->t = 0;
+  c->gepoch++;
   return ME_OK;
 }
 
@@ -653,14 +682,10 @@ static int push_overlapped(me_ctx* c, const uint8_t* cur, const uint8_t* const* 
   return ME_OK;
 }
 
-extern "C" int me_stream_push(me_ctx* c, const uint8_t* cf, int cf_on_host, int16_t* out_qmvs,
-                              uint16_t* out_qsads, int out_on_host, int* n_ref_used) {
-  if (!c || !cf) return ME_EINVAL;
-  if (!cf_on_host && !is_device_ptr(c, cf)) return ME_EINVAL;
-  if (out_qmvs && !out_on_host && !is_device_ptr(c, out_qmvs)) return ME_EINVAL;
-  if (out_qsads && !out_on_host && !is_device_ptr(c, out_qsads)) return ME_EINVAL;
-  int st = stream_alloc(c);
-  if (st != ME_OK) return st;
+// The enqueue body of me_stream_push (arguments validated, ring allocated).
+static int push_enqueue(me_ctx* c, const uint8_t* cf, int cf_on_host, int16_t* out_qmvs, uint16_t* out_qsads,
+                        int out_on_host, int* n_ref_used) {
+  int st;
   c->last_launches = 0;
   c->timed_mask = 0;
   const size_t fb = (size_t)c->W * c->H, sb = (size_t)kNPhase * c->sf_rows * c->sf_pitch;
@@ -752,6 +777,118 @@ extern "C" int me_stream_push(me_ctx* c, const uint8_t* cf, int cf_on_host, int1
   return ME_OK;
 }
 
+// ME_OPT_GRAPH: a device-resident steady-state push (all n_rf RFs present, device frame and
+// outputs, no SF refresh pending) is captured once per ring phase into a CUDA graph and
+// replayed afterwards (SURVEY §8(d) "one CUDA graph per frame").  The ring / SF slots a
+// push uses repeat with period lcm(n_rf + 2, n_rf, 2) (frame ring, SF ring, output parity);
+// a graph is keyed by its phase and the caller's pointers and dropped when any setting
+// changes (gepoch).  The host-side ring bookkeeping of a replayed push is the same as the
+// captured one's, so it is replayed on the host alongside the graph.
+static int graph_period(const me_ctx* c) {
+  auto gcd = [](int a, int b) { while (b) { const int t = a % b; a = b; b = t; } return a; };
+  const int a = ring_slots(c), b = c->n_rf, l = a / gcd(a, b) * b;
+  return l / gcd(l, 2) * 2;
+}
+
+static bool push_needs_sf_refresh(const me_ctx* c) {
+  for (int k = 1; k < c->n_rf; ++k) {
+    const int slot = (int)((c->t - 1 - k) % c->n_rf);
+    if (!(c->sf_v0[slot] <= c->row0 && c->row1 <= c->sf_v1[slot])) return true;
+  }
+  return false;
+}
+
+extern "C" int me_stream_push(me_ctx* c, const uint8_t* cf, int cf_on_host, int16_t* out_qmvs,
+                              uint16_t* out_qsads, int out_on_host, int* n_ref_used) {
+  if (!c || !cf) return ME_EINVAL;
+  if (!cf_on_host && !is_device_ptr(c, cf)) return ME_EINVAL;
+  if (out_qmvs && !out_on_host && !is_device_ptr(c, out_qmvs)) return ME_EINVAL;
+  if (out_qsads && !out_on_host && !is_device_ptr(c, out_qsads)) return ME_EINVAL;
+  int st = stream_alloc(c);
+  if (st != ME_OK) return st;
+  const int period = graph_period(c);
+  const bool graph = c->graph && !cf_on_host && !out_on_host && !c->overlap && !c->pipeline && !c->fuse &&
+                     c->t >= c->n_rf && period <= 64 && !push_needs_sf_refresh(c);
+  if (!graph) return push_enqueue(c, cf, cf_on_host, out_qmvs, out_qsads, out_on_host, n_ref_used);
+  if ((int)c->graphs.size() != period) { graphs_drop(c); c->graphs.resize(period); }
+  me_ctx::Graph& g = c->graphs[c->t % period];
+  const long long t = c->t;
+  const int par = (int)(t & 1);
+  const int slots = ring_slots(c);
+  if (g.exec && g.qm == out_qmvs && g.qs == out_qsads && g.row0 == c->row0 && g.row1 == c->row1 &&
+      g.epoch == c->gepoch && g.timing == c->timing) {
+    // replay: the host bookkeeping push_enqueue did when this phase was captured
+    int y0 = 0, y1 = c->H;
+    if (c->halo_only) {
+      y0 = std::max(0, 16 * c->row0 - c->R - c->max_pmv - 6);
+      y1 = std::min(c->H, 16 * c->row1 + c->R + c->max_pmv + 7);
+    }
+    for (int k = 0; k < c->n_rf; ++k) {
+      const int s = (int)((t - 1 - k) % slots);
+      if (c->fv0[s] > y0 || c->fv1[s] < y1) return ME_ESTATE;
+    }
+    if (g.cf != cf) {                                 // this push's frame: re-point the copy node
+      const size_t off = (size_t)y0 * c->W, len = (size_t)(y1 - y0) * c->W;
+      uint8_t* cur = c->ring + (size_t)(t % slots) * ((size_t)c->W * c->H);
+      if (cudaGraphExecMemcpyNodeSetParams1D(g.exec, g.copy, cur + off, cf + off, len, cudaMemcpyDefault) !=
+          cudaSuccess)
+        return launch_status();
+      g.cf = cf;
+    }
+    if (cudaGraphLaunch(g.exec, c->stream) != cudaSuccess ||
+        cudaEventRecord(c->ev_done[par], c->stream) != cudaSuccess)
+      return launch_status();
+    c->fv0[t % slots] = y0;
+    c->fv1[t % slots] = y1;
+    const int slot = (int)((t - 1) % c->n_rf);
+    c->sf_v0[slot] = c->row0;
+    c->sf_v1[slot] = c->row1;
+    c->last_launches = g.launches;
+    c->timed_mask = g.timed_mask;
+    c->t = t + 1;
+    if (n_ref_used) *n_ref_used = c->n_rf;
+    return ME_OK;
+  }
+  // capture this phase (the timers become external event-record nodes, tmark)
+  if (cudaStreamBeginCapture(c->stream, cudaStreamCaptureModeThreadLocal) != cudaSuccess) return launch_status();
+  c->capturing = true;
+  st = push_enqueue(c, cf, cf_on_host, out_qmvs, out_qsads, out_on_host, n_ref_used);
+  c->capturing = false;
+  cudaGraph_t gr = nullptr;
+  const cudaError_t ec = cudaStreamEndCapture(c->stream, &gr);
+  if (st != ME_OK || ec != cudaSuccess) {
+    if (gr) cudaGraphDestroy(gr);
+    cudaGetLastError();
+    return st != ME_OK ? st : ME_ECUDA;
+  }
+  if (g.exec) { cudaGraphExecDestroy(g.exec); g.exec = nullptr; }
+  if (g.graph) { cudaGraphDestroy(g.graph); g.graph = nullptr; }
+  g.copy = nullptr;
+  size_t nn = 0;
+  cudaGraphGetNodes(gr, nullptr, &nn);
+  std::vector<cudaGraphNode_t> nodes(nn);
+  cudaGraphGetNodes(gr, nodes.data(), &nn);
+  for (cudaGraphNode_t n : nodes) {
+    cudaGraphNodeType ty;
+    if (cudaGraphNodeGetType(n, &ty) == cudaSuccess && ty == cudaGraphNodeTypeMemcpy) g.copy = n;
+  }
+  const cudaError_t ei = g.copy ? cudaGraphInstantiate(&g.exec, gr, 0) : cudaErrorUnknown;
+  if (ei != cudaSuccess) {
+    g.exec = nullptr;
+    cudaGraphDestroy(gr);
+    cudaGetLastError();
+    fprintf(stderr, "feves_me: stream graph: %s\n", cudaGetErrorString(ei));
+    return ME_ECUDA;
+  }
+  g.graph = gr;
+  g.cf = cf; g.qm = out_qmvs; g.qs = out_qsads; g.row0 = c->row0; g.row1 = c->row1;
+  g.epoch = c->gepoch; g.timing = c->timing; g.launches = c->last_launches; g.timed_mask = c->timed_mask;
+  if (cudaGraphLaunch(g.exec, c->stream) != cudaSuccess ||
+      cudaEventRecord(c->ev_done[par], c->stream) != cudaSuccess)   // a real record (the captured one is a node)
+    return launch_status();
+  return ME_OK;
+}
+
 extern "C" int me_sync(me_ctx* c) {
   if (!c) return ME_EINVAL;
   cudaError_t e = cudaStreamSynchronize(c->stream);
@@ -761,6 +898,21 @@ extern "C" int me_sync(me_ctx* c) {
   if (e == cudaSuccess && c->sme_st) e = cudaStreamSynchronize(c->sme_st);
   if (e == cudaSuccess && c->ov_st) e = cudaStreamSynchronize(c->ov_st);
   return e == cudaSuccess ? ME_OK : ME_ECUDA;
+}
+
+// the context stream waits for everything enqueued so far on the internal streams (copy-in,
+// copy-out, INT side stream, SME streams): an event recorded on the context stream after this
+// marks the end of all work of the pushes so far, including the last host download
+extern "C" int me_stream_join(me_ctx* c) {
+  if (!c) return ME_EINVAL;
+  for (cudaStream_t s : {c->copy_in, c->copy_out, c->side, c->sme_st, c->ov_st}) {
+    if (!s) continue;
+    if (!c->ev_switch && cudaEventCreateWithFlags(&c->ev_switch, cudaEventDisableTiming) != cudaSuccess)
+      return launch_status();
+    if (cudaEventRecord(c->ev_switch, s) != cudaSuccess || cudaStreamWaitEvent(c->stream, c->ev_switch, 0) != cudaSuccess)
+      return launch_status();
+  }
+  return ME_OK;
 }
 
 extern "C" int me_stream_outputs(me_ctx* c, int16_t** qmvs, uint16_t** qsads) {
@@ -776,6 +928,7 @@ extern "C" int me_set_timing(me_ctx* c, int on) {
     for (int i = 0; i < 6; ++i)
       if (cudaEventCreate(&c->ev_t[i]) != cudaSuccess) { cudaGetLastError(); return ME_ENOMEM; }
   c->timing = on ? 1 : 0;
+  c->gepoch++;
   return ME_OK;
 }
 
@@ -795,7 +948,9 @@ extern "C" int me_get_timings(me_ctx* c, float* ms_int, float* ms_me, float* ms_
 
 extern "C" int me_set_option(me_ctx* c, int option, int value) {
   if (!c) return ME_EINVAL;
+  c->gepoch++;                                          // cached stream graphs are stale
   switch (option) {
+    case ME_OPT_GRAPH: c->graph = value ? 1 : 0; return ME_OK;
     case ME_OPT_FUSED_SME: c->fuse = value ? 1 : 0; return ME_OK;
     case ME_OPT_PIPELINE_RF: c->pipeline = value ? 1 : 0; return ME_OK;
     case ME_OPT_ME_CTAS_PER_SM:
@@ -803,6 +958,7 @@ extern "C" int me_set_option(me_ctx* c, int option, int value) {
       c->me_ctas_per_sm = value;
       return ME_OK;
     case ME_OPT_SA_INCLUSIVE:
+      if (c->lambda > lambda_limit(c->S, value ? 1 : 0)) return ME_EINVAL;   // 32-bit key (see lambda_limit)
       if (c->stream) cudaStreamSynchronize(c->stream);   // the tables may be in use
       c->inclusive = value ? 1 : 0;
       return upload_key_table(c);
@@ -819,7 +975,7 @@ extern "C" int me_set_option(me_ctx* c, int option, int value) {
       c->overlap = value ? 1 : 0;
       return ME_OK;
     case ME_OPT_LAMBDA:
-      if (value < 0 || value > 2000) return ME_EINVAL;
+      if (value < 0 || value > lambda_limit(c->S, c->inclusive)) return ME_EINVAL;   // 32-bit key
       if (c->stream) cudaStreamSynchronize(c->stream);   // the table may be in use
       c->lambda = value;
       return upload_key_table(c);
@@ -905,7 +1061,6 @@ extern "C" int me_ipc_close(me_ctx* c, void* dptr) {
       if (c->stream) cudaStreamSynchronize(c->stream);   // kernels may still use it
       const cudaError_t e = cudaIpcCloseMemHandle(c->peers[i].base);
       c->peers[i] = {0, 0, nullptr};
-      c->n_checked = 0;                                 // drop cached pointer checks
       return e == cudaSuccess ? ME_OK : ME_ECUDA;
     }
   return ME_EINVAL;
@@ -918,17 +1073,20 @@ extern "C" int me_set_pmv(me_ctx* c, const int16_t* pmv) {
   if (c->max_pmv == 0) return ME_ESTATE;               // the SF margin has no room for a predictor
   if (pmv && !is_device_ptr(c, pmv)) return ME_EINVAL;
   c->d_pmv = pmv;
+  c->gepoch++;
   return ME_OK;
 }
 
-extern "C" int me_mode_decision(me_ctx* c, const int16_t* qmvs, const uint16_t* qsads, int32_t* out_modes) {
-  if (!c || !is_device_ptr(c, qmvs) || !is_device_ptr(c, qsads) || !is_device_ptr(c, out_modes)) return ME_EINVAL;
+extern "C" int me_mode_decision(me_ctx* c, const int16_t* qmvs, const uint16_t* qsads, int n_ref, int32_t* out_modes) {
+  if (!c || n_ref < 1 || n_ref > c->n_rf) return ME_EINVAL;
+  if (!is_device_ptr(c, qmvs) || !is_device_ptr(c, qsads) || !is_device_ptr(c, out_modes)) return ME_EINVAL;
   ModeParams P;
   P.qmvs = reinterpret_cast<const uint32_t*>(qmvs);
   P.sads = qsads;
   P.out = out_modes;
   P.n_mb = (c->row1 - c->row0) * c->mb_cols;
-  P.n_rf = c->n_rf;
+  P.n_rf = n_ref;
+  P.rf_stride = c->n_rf;
   P.lambda = c->lambda;
   P.pmv = c->d_pmv; P.max_pmv = c->max_pmv; P.mb0 = c->row0 * c->mb_cols;
   c->last_launches = 0;

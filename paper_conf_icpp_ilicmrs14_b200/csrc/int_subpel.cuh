@@ -57,8 +57,10 @@ __device__ __forceinline__ uint32_t bytes_of(uint32_t a, uint32_t b) { return __
 
 // One launch, two kinds of blocks (uniform per block, so warps never diverge):
 // blockIdx.z == 1: interior groups [g_lo, g_hi) with no clamping code at all;
-// blockIdx.z == 0: the few border groups, 128 threads = border_bx groups x rows
-// (dispatched first: they are the latency-bound tail otherwise).
+// blockIdx.z == 0: the border groups, 128 threads = border_bx groups x rows per
+// block, blockIdx.x = which border_bx-wide slice of the border groups (every
+// border group is covered: all of them when W % 4 != 0 or the RF rows are not
+// 4-byte aligned; dispatched first: they are the latency-bound tail otherwise).
 template <bool INTERIOR>
 __device__ __forceinline__ void int_body(const IntParams& P, int g, int rr) {
   const int x0 = 16 * g - P.pad, y = rr - P.pad;
@@ -187,10 +189,9 @@ __global__ void __launch_bounds__(128, FEVES_INT_MINB) int_subpel_kernel(const I
     const int rr = P.row_begin + blockIdx.y * blockDim.y + threadIdx.y;
     if (g < P.g_hi && rr < P.row_end) int_body<true>(P, g, rr);
   } else {
-    if (blockIdx.x != 0) return;
     const int t = threadIdx.y * blockDim.x + threadIdx.x;
     const int bx = P.border_bx, by = (blockDim.x * blockDim.y) / bx;
-    const int tb = t % bx, tr = t / bx;
+    const int tb = blockIdx.x * bx + t % bx, tr = t / bx;
     const int groups = P.pitch / 16, nb = groups - (P.g_hi - P.g_lo);
     if (tb >= nb) return;
     const int g = tb < P.g_lo ? tb : P.g_hi + (tb - P.g_lo);

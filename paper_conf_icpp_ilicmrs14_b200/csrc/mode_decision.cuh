@@ -15,7 +15,8 @@ struct ModeParams {
   const uint32_t* qmvs;     // [mb][n_rf][41] packed int16 pairs (sme output)
   const uint16_t* sads;
   int32_t* out;             // [mb][10]: mb_type, sub_type[4], ref per 8x8 [4], cost
-  int n_mb, n_rf, lambda;
+  int n_mb, n_rf, lambda;   // n_rf = valid RF slots searched (<= rf_stride)
+  int rf_stride;            // RF dimension of the layout (the context's n_rf)
   const int16_t* pmv;       // G21 predictor [frame MB][n_rf][2] or null; MB i of the arrays = frame MB mb0 + i
   int max_pmv, mb0;
 };
@@ -24,13 +25,13 @@ __global__ void __launch_bounds__(128) mode_decision_kernel(const ModeParams P) 
   const int i = blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= P.n_mb) return;
   auto J = [&](int r, int p) -> int {
-    const size_t o = ((size_t)i * P.n_rf + r) * kNPart + p;
+    const size_t o = ((size_t)i * P.rf_stride + r) * kNPart + p;
     int j = P.sads[o];
     if (P.lambda) {
       const uint32_t mv = P.qmvs[o];
       int qpx = 0, qpy = 0;                  // G21: rate against 4p
       if (P.pmv) {
-        const size_t pi = ((size_t)(P.mb0 + i) * P.n_rf + r) * 2;
+        const size_t pi = ((size_t)(P.mb0 + i) * P.rf_stride + r) * 2;
         qpx = 4 * min(max((int)P.pmv[pi], -P.max_pmv), P.max_pmv);
         qpy = 4 * min(max((int)P.pmv[pi + 1], -P.max_pmv), P.max_pmv);
       }

@@ -38,6 +38,7 @@ struct SmeParams {
   const int16_t* pmv;                                 // G21 predictor [frame MB][rf_stride][2] or null
   int max_pmv;
   int fence;                                          // outputs are peer memory (me_ipc_open): system fence at exit
+  int cf_vec;                                         // W % 4 == 0 and cf 4-byte aligned: CF rows as aligned words
   uint32_t k_hi;                                      // = kAvgHi (vavg4)
 };
 
@@ -290,7 +291,7 @@ __device__ __forceinline__ void refine_mode(const SmeParams& P, const uint8_t* _
     }
     const int yg = ys0 + 4 * g * YG;   // first frame row of this group
     uint32_t cf[4 * YG];               // this group's CF strip rows
-    if ((P.W & 3) == 0 && xs + 3 < P.W && yg + 4 * YG <= P.H) {   // inside the frame: aligned words
+    if (P.cf_vec && xs + 3 < P.W && yg + 4 * YG <= P.H) {        // inside the frame: aligned words
       const uint32_t* c0 = reinterpret_cast<const uint32_t*>(P.cf + (size_t)yg * P.W + xs);
 #pragma unroll
       for (int r = 0; r < 4 * YG; ++r) cf[r] = __ldg(c0 + r * (P.W >> 2));

@@ -74,3 +74,18 @@ def test_create_pmv_rejects_bad_arguments(feves_lib, args):
     assert not feves_lib.me_create_pmv(*args)
     assert feves_lib.me_last_error() == -1
     assert feves_lib.me_set_pmv(None, None) == -1
+
+
+@pytest.mark.parametrize("S,inc,lmax", [(128, 0, 1731), (128, 1, 1731), (64, 0, 1935), (64, 1, 1935),
+                                        (32, 0, 2000), (4, 0, 2000)])
+def test_lambda_limit_keeps_the_key_exact(feves_lib, S, inc, lmax):
+    """the ME key J * 2^15 + rank is 32 bits, so J = SAD + lambda * R must stay
+    below 2^17.  Hand-derived bounds: max R = 2 * se(4 * 64) = 2 * 19 bits at S = 128 (and for
+    the inclusive +64), 2 * se(4 * 32) = 2 * 17 at S = 64: 65280 + 1731 * 38 = 131058 < 131072 <
+    65280 + 1732 * 38; 65280 + 1935 * 34 = 131070 < 131072.  Smaller SAs stay at the API cap 2000."""
+    Sc = S + inc
+    ka = (ctypes.c_uint32 * (Sc * ((Sc + 3) & ~3)))()
+    inv = (ctypes.c_uint32 * ((S + 1) ** 2))()
+    glob = (ctypes.c_uint32 * (4 * 4096))()
+    assert feves_lib.me_key_tables(S, inc, lmax, ka, inv, glob) == 0
+    assert feves_lib.me_key_tables(S, inc, lmax + 1, ka, inv, glob) == -1

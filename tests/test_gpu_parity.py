@@ -492,3 +492,44 @@ def test_stream_overlap_sme_equals_serial(feves, host):
         np.testing.assert_array_equal(qa, qb)
         np.testing.assert_array_equal(sa, sb)
     assert any(u == n_rf for _, _, u in a)
+
+
+@pytest.mark.parametrize("n_rf,halo", [(2, False), (4, True)])
+def test_stream_graph_replay_equals_oracle(feves, orc, n_rf, halo):
+    """ME_OPT_GRAPH (SURVEY §8(d) one CUDA graph per frame): steady-state pushes are captured
+    once per ring phase (period lcm(n_rf+2, n_rf, 2)) and REPLAYED; the frames come from 5
+    distinct device tensors (the graph's copy node is re-pointed) into ONE output buffer, and
+    a stripe change mid-stream re-captures.  Every frame's outputs == the oracle."""
+    W, H, S = 80, 64, 16
+    frames = [gen_tex(W, H, t, 83) for t in range(3 * (n_rf + 2) * n_rf + 4)]
+    dev = [_dev(f) for f in frames[:5]]
+    me = feves.MotionEstimator(W, H, S, n_rf)
+    me.set_option(me.OPT_GRAPH, 1)
+    if halo:
+        me.set_option(me.OPT_HALO_ONLY, 1)
+        me.set_rows(1, 3)
+    out = me.new_mvs()
+    n_checked = 0
+    for t, f in enumerate(frames):
+        src = dev[t % 5]
+        src.copy_(_dev(f))                               # torch stream == context stream: ordered
+        if t == len(frames) - 3 and not halo:
+            me.set_rows(1, 4)                            # re-capture with another stripe
+            out = me.new_mvs()
+        qm, qs, used = me.stream_push(src, out=out)
+        if used < n_rf and t > n_rf:
+            raise AssertionError("ramp")
+        if t % 3 == 0 or t >= len(frames) - 4:           # oracle on a subset of the frames
+            torch.cuda.synchronize()
+            rfs = [frames[t - 1 - k] for k in range(used)]
+            mbs = orc.all_mbs(W, H, me.row0, me.row1)
+            if not used:
+                continue
+            o_m, _ = orc.me(f, rfs, S, mb_list=mbs)
+            o_q, o_s = orc.sme(f, rfs, o_m, mb_list=mbs)
+            n = len(mbs)
+            np.testing.assert_array_equal(qm.cpu().numpy().reshape(n, n_rf, 41, 2)[:, :used], o_q, err_msg=str(t))
+            np.testing.assert_array_equal(qs.cpu().numpy().reshape(n, n_rf, 41)[:, :used], o_s, err_msg=str(t))
+            n_checked += 1
+    assert n_checked >= 8
+    me.close()
