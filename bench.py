@@ -51,7 +51,8 @@ def parse():
                     help="reference arm: seconds of oracle wall time per step (a seeded MB sample)")
     ap.add_argument("--cpu-frame", choices=["full", "sample"], default="full",
                     help="cpu_baseline: the oracle on ONE FULL frame on all host cores (default) or a sample")
-    ap.add_argument("--graph", type=int, default=1, help="ME_OPT_GRAPH: one CUDA graph per frame (default 1)")
+    ap.add_argument("--graph", type=int, default=1,
+                    help="ME_OPT_GRAPH: one CUDA graph per frame (default 1; 0 = multi-stream enqueue)")
     ap.add_argument("--pipeline", type=int, default=None, help="ME_OPT_PIPELINE_RF (default: library default)")
     ap.add_argument("--me-ctas", type=int, default=None, help="ME_OPT_ME_CTAS_PER_SM")
     ap.add_argument("--fused", type=int, default=None, help="ME_OPT_FUSED_SME")
@@ -75,6 +76,14 @@ def peaks():
         return {"hbm_gbs": 6650.0, "sm_max_mhz": 1965.0}, "fallback"
 
 
+def graph_period(n_rf):
+    """ring phases of me_stream_push (ME_OPT_GRAPH captures one graph per phase):
+    lcm(n_rf + 2 frame slots, n_rf SF slots, 2 output buffers)"""
+    import math
+    a = (n_rf + 2) * n_rf // math.gcd(n_rf + 2, n_rf)
+    return a * 2 // math.gcd(a, 2)
+
+
 def workload_units(cfg, n_ref=None):
     """Algorithmic work of one frame."""
     mbc, mbr = -(-cfg.width // 16), -(-cfg.height // 16)
@@ -90,8 +99,14 @@ def workload_units(cfg, n_ref=None):
 
 
 class Clocks:
-    """nvidia-smi sampler for the timed region (B200_PROFILING.md clocks line)."""
+    """SM clock + throttle-reason sampler for the timed region (B200_PROFILING.md clocks line):
+    an NVML thread polling every 2 ms (the timed region of a default run lasts only ~20-30 ms),
+    nvidia-smi -lms 50 when NVML is unavailable."""
 
+    NAMES = {"hw_slowdown": "nvmlClocksEventReasonHwSlowdown",
+             "hw_thermal_slowdown": "nvmlClocksEventReasonHwThermalSlowdown",
+             "sw_thermal_slowdown": "nvmlClocksEventReasonSwThermalSlowdown",
+             "sw_power_cap": "nvmlClocksEventReasonSwPowerCap"}
     Q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
          "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
          "clocks_event_reasons.sw_power_cap")
@@ -99,8 +114,35 @@ class Clocks:
     def __init__(self, index):
         self.index = index
         self.p = None
+        self.th = None
+        self.samples, self.mx, self.reasons = [], None, set()
 
     def start(self):
+        import threading
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            h = pynvml.nvmlDeviceGetHandleByIndex(self.index)
+            self.mx = float(pynvml.nvmlDeviceGetMaxClockInfo(h, pynvml.NVML_CLOCK_SM))
+            self.stop_ev = threading.Event()
+
+            def run():
+                while not self.stop_ev.is_set():
+                    try:
+                        self.samples.append(float(pynvml.nvmlDeviceGetClockInfo(h, pynvml.NVML_CLOCK_SM)))
+                        r = pynvml.nvmlDeviceGetCurrentClocksEventReasons(h)
+                        for n, attr in self.NAMES.items():
+                            if r & getattr(pynvml, attr):
+                                self.reasons.add(n)
+                    except pynvml.NVMLError:
+                        pass
+                    self.stop_ev.wait(0.002)
+            self.th = threading.Thread(target=run, daemon=True)
+            self.th.start()
+            time.sleep(0.01)
+            return
+        except Exception:
+            self.th = None
         try:
             self.p = subprocess.Popen(["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.Q}",
                                        "--format=csv,noheader,nounits", "-lms", "50"],
@@ -110,12 +152,19 @@ class Clocks:
             self.p = None
 
     def stop(self):
+        if self.th is not None:
+            self.stop_ev.set()
+            self.th.join()
+            sm = self.samples
+            busy = [x for x in sm if x > 300] or sm
+            return {"sm_mhz": statistics.median(busy) if busy else None, "sm_max_mhz": self.mx,
+                    "reasons": sorted(self.reasons), "samples": len(sm), "sampler": "nvml 2 ms"}
         if self.p is None:
             return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
         self.p.terminate()
         out, _ = self.p.communicate(timeout=10)
         sm, mx, reasons = [], None, set()
-        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        names = list(self.NAMES)
         for line in out.strip().splitlines():
             f = [x.strip() for x in line.split(",")]
             if len(f) < 7:
@@ -130,7 +179,7 @@ class Clocks:
                     reasons.add(n)
         busy = [s for s in sm if s > 300] or sm
         return {"sm_mhz": statistics.median(busy) if busy else None, "sm_max_mhz": mx,
-                "reasons": sorted(reasons), "samples": len(sm)}
+                "reasons": sorted(reasons), "samples": len(sm), "sampler": "nvidia-smi 50 ms"}
 
 
 # ----------------------------------------------------------------- reference --
@@ -323,35 +372,62 @@ def run_feves(args, cfg):
     out_dev = me.new_mvs()
     me.stream_reset()
     t = 0
-    while t < cfg.n_rf + args.warmup:        # fill the RF/SF ring (P:323 ramp), then warm up
+    # fill the RF/SF ring (P:323 ramp), capture every ring phase's graph (period lcm(n_rf+2, n_rf, 2)),
+    # then the W untimed warm-up steps
+    n_fill = cfg.n_rf + (2 * graph_period(cfg.n_rf) if args.graph and world == 1 else 0)
+    while t < n_fill + args.warmup:
         push(t)
         t += 1
     torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
 
-    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
-    mod = []
-    launches = 0
+    def timed(n, timers):
+        """n steps, each bracketed by CUDA events on the stream the push runs on, L2 flushed
+        before each; timers: the library's per-module CUDA-event timers on (one host sync per
+        step to read them) or off (no instrumentation inside the step)"""
+        nonlocal t
+        me.set_timing(timers)
+        ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(n)]
+        mods, launches = [], 0
+        for k in range(n):
+            flush.fill_(k & 0xff)
+            ev[k][0].record(stream)
+            push(t)
+            ev[k][1].record(stream)
+            t += 1
+            if timers:
+                mods.append(me.timings())        # waits for this step's module events
+            launches += me.launches
+        torch.cuda.synchronize()
+        return [a.elapsed_time(b) for a, b in ev], mods, launches
+
+    # value: K steps without instrumentation; kernels_ms / roofline: a second pass with the
+    # per-module timers (the events cost a few us per step, so they stay out of `value`)
     clocks = Clocks(local)
     clocks.start()
-    for k in range(args.steps):
-        flush.fill_(k & 0xff)
-        ev[k][0].record(stream)
-        push(t)
-        ev[k][1].record(stream)
-        t += 1
-        mod.append(me.timings())             # waits for this step's module events
-        launches += me.launches
-    torch.cuda.synchronize()
+    step_ms, _, launches = timed(args.steps, False)
     ck = clocks.stop()
-    step_ms = [a.elapsed_time(b) for a, b in ev]
     tot = torch.tensor([sum(step_ms)], dtype=torch.float64, device=dev)
     if world > 1:
         tot = _all_max(tot)
         dist.barrier()
     total_ms = float(tot.item())
     fps = args.steps / (total_ms / 1e3)
+    mod_ms, mod, _ = timed(max(5, min(args.steps, 20)), True)
+    graph_ab = None
+    if world == 1:                                   # the other ME_OPT_GRAPH setting, same protocol
+        me.set_option(me.OPT_GRAPH, 0 if args.graph else 1)
+        for _ in range(2 * graph_period(cfg.n_rf)):  # warm-up: capture every ring phase
+            push(t)
+            t += 1
+        alt_ms, _, _ = timed(max(5, min(args.steps, 20)), False)
+        me.set_option(me.OPT_GRAPH, args.graph)
+        graph_ab = {("stream_ms_per_step" if args.graph else "graph_ms_per_step"): statistics.mean(alt_ms),
+                    ("graph_ms_per_step" if args.graph else "stream_ms_per_step"): total_ms / args.steps,
+                    "note": "one CUDA graph per frame (ME_OPT_GRAPH: INT || ME -> SME, frame copy and fork/join "
+                            "captured once per ring phase and replayed) vs the multi-stream enqueue; the faster "
+                            "one is the bench default (--graph)"}
 
     # INT in isolation (inside the step it overlaps ME on the side stream, P:86); the
     # library's own module timers are switched off so only the outer events bracket it
@@ -512,6 +588,7 @@ def run_feves(args, cfg):
                            "; fused: INT(t-1) then one ME+SME kernel" if fused else
                            "; INT runs concurrently with ME (P:86) on a side stream")},
         "clocks": ck,
+        "graph_ab": graph_ab,
         "e2e": e2e,
         "gpu_launches": launches,
         "roofline": {"bound": "alu", "kernel": "me_fsbm_kernel<64,fused>" if fused else "me_fsbm_kernel<64>",

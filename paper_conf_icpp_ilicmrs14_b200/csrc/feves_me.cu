@@ -229,6 +229,16 @@ static int upload_key_table(me_ctx* c) {
 }
 
 // ------------------------------------------------------------ lifetime ----
+// The context's own stream runs at the highest priority and the INT side stream at the
+// lowest: INT (concurrent with ME) then only takes SMs that ME's CTAs leave free, i.e. it
+// fills ME's last-wave tail instead of delaying ME's first wave.  Stream-captured graphs keep
+// these as per-node priorities (cudaGraphInstantiateFlagUseNodePriority).
+static cudaError_t create_own_stream(me_ctx* c) {
+  int least = 0, greatest = 0;
+  cudaDeviceGetStreamPriorityRange(&least, &greatest);
+  return cudaStreamCreateWithPriority(&c->own, cudaStreamNonBlocking, greatest);
+}
+
 extern "C" me_ctx* me_create(int width, int height, int sa_range, int n_rf) {
   return me_create_pmv(width, height, sa_range, n_rf, 0);
 }
@@ -266,7 +276,7 @@ extern "C" me_ctx* me_create_pmv(int width, int height, int sa_range, int n_rf, 
             cudaMalloc(&c->d_glob, (size_t)4 * 4096 * 4) == cudaSuccess &&
             cudaMalloc(&c->d_mvs, nmv * 4) == cudaSuccess &&
             cudaMalloc(&c->d_sads, nmv * 2) == cudaSuccess &&
-            cudaStreamCreateWithFlags(&c->own, cudaStreamNonBlocking) == cudaSuccess;
+            create_own_stream(c) == cudaSuccess;
   if (ok) {
     c->stream = c->own;
     ok = upload_key_table(c) == ME_OK &&
@@ -471,7 +481,7 @@ static int launch_int(me_ctx* c, const uint8_t* rf, uint8_t* sf, cudaStream_t st
 
 static int launch_sme(me_ctx* c, const uint8_t* cf, const uint8_t* const* sfs, const int16_t* in_mvs,
                       const uint16_t* in_sads, int16_t* out_qmvs, uint16_t* out_sads, int n_ref, cudaStream_t st,
-                      int rf0 = 0) {
+                      int rf0 = 0, int marks = 3) {   // marks: bit 0 = start timer event, bit 1 = stop
   SmeParams P;
   memset(&P, 0, sizeof(P));
   P.cf = cf;
@@ -492,11 +502,11 @@ static int launch_sme(me_ctx* c, const uint8_t* cf, const uint8_t* const* sfs, c
   P.cf_vec = (c->W % 4 == 0) && ((reinterpret_cast<uintptr_t>(cf) & 3) == 0);   // aligned CF word loads
   P.k_hi = kAvgHi;
   const int warps = n_ref * P.n_rows * P.groups;
-  tmark(c, 4, st);
+  if (marks & 1) tmark(c, 4, st);
   const dim3 sg((warps + 3) / 4, 7);   // y = partition mode
   const cudaError_t e = sme_launch(c->lambda != 0, c->satd != 0, sg, 128, st, P);
   if (e != cudaSuccess) { fprintf(stderr, "feves_me: SME launch: %s\n", cudaGetErrorString(e)); return ME_ECUDA; }
-  tmark(c, 5, st);
+  if (marks & 2) tmark(c, 5, st);
   c->last_launches++;
   return launch_status();
 }
@@ -623,7 +633,7 @@ static int stream_alloc(me_ctx* c) {
   bool ok = cudaMalloc(&c->ring, fb * ring_slots(c)) == cudaSuccess &&
             cudaMalloc(&c->sf_ring, sb * c->n_rf) == cudaSuccess && cudaMalloc(&c->d_qmvs, nmv * 4) == cudaSuccess &&
             cudaMalloc(&c->d_qsads, nmv * 2) == cudaSuccess &&
-            cudaStreamCreateWithFlags(&c->side, cudaStreamNonBlocking) == cudaSuccess &&
+            cudaStreamCreateWithPriority(&c->side, cudaStreamNonBlocking, 0 /* lowest */) == cudaSuccess &&
             cudaStreamCreateWithFlags(&c->copy_in, cudaStreamNonBlocking) == cudaSuccess &&
             cudaStreamCreateWithFlags(&c->copy_out, cudaStreamNonBlocking) == cudaSuccess &&
             cudaEventCreateWithFlags(&c->ev_fork, cudaEventDisableTiming) == cudaSuccess &&
@@ -764,9 +774,15 @@ static int push_enqueue(me_ctx* c, const uint8_t* cf, int cf_on_host, int16_t* o
     const size_t nmv = (size_t)(c->row1 - c->row0) * c->mb_cols * c->n_rf * kNPart;
     if (cudaEventRecord(c->ev_done[par], c->ov_pending ? c->ov_st : c->stream) != cudaSuccess) return launch_status();
     if (out_on_host) {   // download on the copy-out stream, overlapping the next frame's compute
+      // only the n_ref searched RF slots of every MB (slots >= n_ref stay untouched, as for
+      // device outputs): one 2-D copy, rows = MBs, pitch = n_rf slots
+      const size_t n_mb = nmv / ((size_t)c->n_rf * kNPart), slot = (size_t)kNPart;
+      const size_t pm = (size_t)c->n_rf * slot * 4, ps = (size_t)c->n_rf * slot * 2;
       if (cudaStreamWaitEvent(c->copy_out, c->ev_done[par], 0) != cudaSuccess ||
-          (out_qmvs && cudaMemcpyAsync(out_qmvs, qm, nmv * 4, cudaMemcpyDeviceToHost, c->copy_out) != cudaSuccess) ||
-          (out_qsads && cudaMemcpyAsync(out_qsads, qs, nmv * 2, cudaMemcpyDeviceToHost, c->copy_out) != cudaSuccess) ||
+          (out_qmvs && cudaMemcpy2DAsync(out_qmvs, pm, qm, pm, (size_t)n_ref * slot * 4, n_mb, cudaMemcpyDeviceToHost,
+                                         c->copy_out) != cudaSuccess) ||
+          (out_qsads && cudaMemcpy2DAsync(out_qsads, ps, qs, ps, (size_t)n_ref * slot * 2, n_mb, cudaMemcpyDeviceToHost,
+                                          c->copy_out) != cudaSuccess) ||
           cudaEventRecord(c->ev_down[par], c->copy_out) != cudaSuccess)
         return launch_status();
     }
@@ -798,6 +814,9 @@ static bool push_needs_sf_refresh(const me_ctx* c) {
   return false;
 }
 
+static int push_graph(me_ctx* c, const uint8_t* cf, int16_t* out_qmvs, uint16_t* out_qsads, int* n_ref_used,
+                      int period);
+
 extern "C" int me_stream_push(me_ctx* c, const uint8_t* cf, int cf_on_host, int16_t* out_qmvs,
                               uint16_t* out_qsads, int out_on_host, int* n_ref_used) {
   if (!c || !cf) return ME_EINVAL;
@@ -810,6 +829,12 @@ extern "C" int me_stream_push(me_ctx* c, const uint8_t* cf, int cf_on_host, int1
   const bool graph = c->graph && !cf_on_host && !out_on_host && !c->overlap && !c->pipeline && !c->fuse &&
                      c->t >= c->n_rf && period <= 64 && !push_needs_sf_refresh(c);
   if (!graph) return push_enqueue(c, cf, cf_on_host, out_qmvs, out_qsads, out_on_host, n_ref_used);
+  return push_graph(c, cf, out_qmvs, out_qsads, n_ref_used, period);
+}
+
+static int push_graph(me_ctx* c, const uint8_t* cf, int16_t* out_qmvs, uint16_t* out_qsads, int* n_ref_used,
+                      int period) {
+  int st;
   if ((int)c->graphs.size() != period) { graphs_drop(c); c->graphs.resize(period); }
   me_ctx::Graph& g = c->graphs[c->t % period];
   const long long t = c->t;
@@ -849,13 +874,21 @@ extern "C" int me_stream_push(me_ctx* c, const uint8_t* cf, int cf_on_host, int1
     if (n_ref_used) *n_ref_used = c->n_rf;
     return ME_OK;
   }
-  // capture this phase (the timers become external event-record nodes, tmark)
-  if (cudaStreamBeginCapture(c->stream, cudaStreamCaptureModeThreadLocal) != cudaSuccess) return launch_status();
+  // capture this phase on the context's own stream (capturable even when the caller's is the
+  // legacy default stream; nothing executes during a capture, so no ordering is needed), then
+  // launch it on the caller's stream (the timers become external event-record nodes, tmark)
+  cudaStream_t caller = c->stream;
+  c->stream = c->own;
+  if (cudaStreamBeginCapture(c->stream, cudaStreamCaptureModeThreadLocal) != cudaSuccess) {
+    c->stream = caller;
+    return launch_status();
+  }
   c->capturing = true;
-  st = push_enqueue(c, cf, cf_on_host, out_qmvs, out_qsads, out_on_host, n_ref_used);
+  st = push_enqueue(c, cf, 0, out_qmvs, out_qsads, 0, n_ref_used);
   c->capturing = false;
   cudaGraph_t gr = nullptr;
   const cudaError_t ec = cudaStreamEndCapture(c->stream, &gr);
+  c->stream = caller;
   if (st != ME_OK || ec != cudaSuccess) {
     if (gr) cudaGraphDestroy(gr);
     cudaGetLastError();
@@ -872,7 +905,7 @@ extern "C" int me_stream_push(me_ctx* c, const uint8_t* cf, int cf_on_host, int1
     cudaGraphNodeType ty;
     if (cudaGraphNodeGetType(n, &ty) == cudaSuccess && ty == cudaGraphNodeTypeMemcpy) g.copy = n;
   }
-  const cudaError_t ei = g.copy ? cudaGraphInstantiate(&g.exec, gr, 0) : cudaErrorUnknown;
+  const cudaError_t ei = g.copy ? cudaGraphInstantiate(&g.exec, gr, cudaGraphInstantiateFlagUseNodePriority) : cudaErrorUnknown;
   if (ei != cudaSuccess) {
     g.exec = nullptr;
     cudaGraphDestroy(gr);
