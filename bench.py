@@ -51,6 +51,7 @@ def parse():
                     help="reference arm: seconds of oracle wall time per step (a seeded MB sample)")
     ap.add_argument("--cpu-frame", choices=["full", "sample"], default="full",
                     help="cpu_baseline: the oracle on ONE FULL frame on all host cores (default) or a sample")
+    ap.add_argument("--sme-kernel", type=int, default=None, help="ME_OPT_SME_KERNEL (0 global-load, 1 staged)")
     ap.add_argument("--graph", type=int, default=1,
                     help="ME_OPT_GRAPH: one CUDA graph per frame (default 1; 0 = multi-stream enqueue)")
     ap.add_argument("--pipeline", type=int, default=None, help="ME_OPT_PIPELINE_RF (default: library default)")
@@ -344,7 +345,8 @@ def run_feves(args, cfg):
     r0, r1 = stripes(me.mb_rows, world)[rank]
     me.set_rows(r0, r1)      # (ShardedStream may re-split later in adaptive mode)
     for opt, val in ((me.OPT_PIPELINE_RF, args.pipeline), (me.OPT_ME_CTAS_PER_SM, args.me_ctas),
-                     (me.OPT_FUSED_SME, args.fused), (me.OPT_GRAPH, args.graph if world == 1 else None)):
+                     (me.OPT_FUSED_SME, args.fused), (me.OPT_GRAPH, args.graph if world == 1 else None),
+                     (me.OPT_SME_KERNEL, args.sme_kernel)):
         if val is not None:
             me.set_option(opt, val)
     me.set_timing(True)

@@ -17,6 +17,7 @@
 
 #include "int_subpel.cuh"
 #include "launch.cuh"   // ME / SME launches (their own translation units: me_s*.cu, sme.cu)
+#include "sme_smem.cuh"  // kSme2Mb (staged SME group size)
 #include "mode_decision.cuh"
 
 using namespace feves;
@@ -94,6 +95,8 @@ struct me_ctx {
   };
   std::vector<Graph> graphs;
   int graph;             // ME_OPT_GRAPH
+  int sme_kernel;        // ME_OPT_SME_KERNEL: 0 global-load SME (default), 1 shared-memory staged
+  int* d_ovf;            // staged SME overflow list: [0] count, then (MB, RF) items
   bool capturing;        // push_enqueue runs inside a stream capture
   long long gepoch;      // bumped by every setting change: cached graphs are stale
 };
@@ -276,10 +279,12 @@ extern "C" me_ctx* me_create_pmv(int width, int height, int sa_range, int n_rf, 
             cudaMalloc(&c->d_glob, (size_t)4 * 4096 * 4) == cudaSuccess &&
             cudaMalloc(&c->d_mvs, nmv * 4) == cudaSuccess &&
             cudaMalloc(&c->d_sads, nmv * 2) == cudaSuccess &&
+            cudaMalloc(&c->d_ovf, (1 + (size_t)c->mb_cols * c->mb_rows * n_rf) * sizeof(int)) == cudaSuccess &&
             create_own_stream(c) == cudaSuccess;
   if (ok) {
     c->stream = c->own;
-    ok = upload_key_table(c) == ME_OK &&
+    c->sme_kernel = 0;   // the staged SME measured on par (145-149 vs 145 us at 1080p S64 4 RF): opt-in
+    ok = upload_key_table(c) == ME_OK && sme2_init() == cudaSuccess &&
          set_me_smem(200 * 1024) == cudaSuccess;   // max; the launch asks for what it needs
   }
   if (!ok) {
@@ -305,6 +310,7 @@ extern "C" void me_destroy(me_ctx* c) {
   cudaFree(c->d_glob);
   cudaFree(c->d_mvs);
   cudaFree(c->d_sads);
+  cudaFree(c->d_ovf);
   cudaFree(c->ring);
   cudaFree(c->sf_ring);
   cudaFree(c->d_qmvs);
@@ -503,11 +509,21 @@ static int launch_sme(me_ctx* c, const uint8_t* cf, const uint8_t* const* sfs, c
   P.k_hi = kAvgHi;
   const int warps = n_ref * P.n_rows * P.groups;
   if (marks & 1) tmark(c, 4, st);
-  const dim3 sg((warps + 3) / 4, 7);   // y = partition mode
-  const cudaError_t e = sme_launch(c->lambda != 0, c->satd != 0, sg, 128, st, P);
+  // shared-memory staged SME (sme_smem.cuh) for the SAD distortion with the ME SADs given
+  // and 16-byte aligned SFs (cp.async); the global-load kernel otherwise
+  bool staged = c->sme_kernel == 1 && !c->satd && in_sads != nullptr;
+  for (int k = 0; k < n_ref; ++k) staged = staged && ((reinterpret_cast<uintptr_t>(sfs[k]) & 15) == 0);
+  cudaError_t e;
+  if (staged) {
+    e = sme2_launch(c->lambda != 0, n_ref * P.n_rows * ((c->mb_cols + kSme2Mb - 1) / kSme2Mb), st, P, c->d_ovf);
+    c->last_launches += 2;
+  } else {
+    const dim3 sg((warps + 3) / 4, 7);   // y = partition mode
+    e = sme_launch(c->lambda != 0, c->satd != 0, sg, 128, st, P);
+    c->last_launches++;
+  }
   if (e != cudaSuccess) { fprintf(stderr, "feves_me: SME launch: %s\n", cudaGetErrorString(e)); return ME_ECUDA; }
   if (marks & 2) tmark(c, 5, st);
-  c->last_launches++;
   return launch_status();
 }
 
@@ -984,6 +1000,10 @@ extern "C" int me_set_option(me_ctx* c, int option, int value) {
   c->gepoch++;                                          // cached stream graphs are stale
   switch (option) {
     case ME_OPT_GRAPH: c->graph = value ? 1 : 0; return ME_OK;
+    case ME_OPT_SME_KERNEL:
+      if (value < 0 || value > 1) return ME_EINVAL;
+      c->sme_kernel = value;
+      return ME_OK;
     case ME_OPT_FUSED_SME: c->fuse = value ? 1 : 0; return ME_OK;
     case ME_OPT_PIPELINE_RF: c->pipeline = value ? 1 : 0; return ME_OK;
     case ME_OPT_ME_CTAS_PER_SM:
@@ -1097,6 +1117,15 @@ extern "C" int me_ipc_close(me_ctx* c, void* dptr) {
       return e == cudaSuccess ? ME_OK : ME_ECUDA;
     }
   return ME_EINVAL;
+}
+
+extern "C" int me_sme_overflow_count(me_ctx* c) {
+  if (!c) return ME_EINVAL;
+  int n = 0;
+  if (cudaStreamSynchronize(c->stream) != cudaSuccess ||
+      cudaMemcpy(&n, c->d_ovf, sizeof(int), cudaMemcpyDeviceToHost) != cudaSuccess)
+    return launch_status();
+  return n;
 }
 
 extern "C" int me_set_fused(me_ctx* c, int on) { return me_set_option(c, ME_OPT_FUSED_SME, on); }

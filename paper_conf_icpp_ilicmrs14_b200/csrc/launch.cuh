@@ -67,5 +67,10 @@ FEVES_ME_TU_DECL(128)
 
 // SME (sme.cu): rd = rate term compiled in (G18), satd = Hadamard distortion (G20)
 cudaError_t sme_launch(bool rd, bool satd, dim3 grid, int threads, cudaStream_t st, const SmeParams& P);
+// SME with shared-memory staged windows (sme_smem.cuh), one CTA per group of 8 MBs x RF:
+// ovf = device int[1 + n_groups] overflow list (counter reset here), then the global-load
+// kernel on the overflow groups
+cudaError_t sme2_launch(bool rd, int n_groups, cudaStream_t st, const SmeParams& P, int* ovf);
+cudaError_t sme2_init();   // dynamic shared-memory attribute (once per process/device)
 
 }  // namespace feves

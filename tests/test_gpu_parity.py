@@ -533,3 +533,26 @@ def test_stream_graph_replay_equals_oracle(feves, orc, n_rf, halo):
             n_checked += 1
     assert n_checked >= 8
     me.close()
+
+
+@pytest.mark.parametrize("lam,S,kind", [(0, 64, "tex"), (0, 32, "noise"), (7, 16, "flat"), (0, 128, "tex")])
+def test_sme_staged_kernel_equals_oracle(feves, orc, lam, S, kind):
+    """ME_OPT_SME_KERNEL = 1: the shared-memory staged SME (TMA-staged sub-pel footprint box per
+    8-MB group; boxes beyond the region through the overflow list) == oracle, with and without
+    the rate term, on frames wide enough for several groups and a ragged last group"""
+    W, H, n_rf = 200, 72, 2                              # 13 MBs per row: groups of 8 + 5
+    cf, rfs = _frames(kind, W, H, n_rf, 91 + S + lam)
+    me = feves.MotionEstimator(W, H, S, n_rf)
+    me.set_option(me.OPT_SME_KERNEL, 1)
+    if lam:
+        me.set_lambda(lam)
+    tcf, trfs = _dev(cf), [_dev(r) for r in rfs]
+    sfs = [me.new_sf() for _ in trfs]
+    (m, s), (q, qs) = me.encode_frame(tcf, trfs, sfs, n_int=n_rf, out_me=me.new_mvs())
+    torch.cuda.synchronize()
+    n = me.mb_rows * me.mb_cols
+    o_m, _ = orc.me(cf, rfs, S, lam=lam)
+    o_q, o_qs = orc.sme(cf, rfs, o_m, lam=lam)
+    np.testing.assert_array_equal(q.cpu().numpy().reshape(n, n_rf, 41, 2), o_q)
+    np.testing.assert_array_equal(qs.cpu().numpy().reshape(n, n_rf, 41), o_qs)
+    me.close()
