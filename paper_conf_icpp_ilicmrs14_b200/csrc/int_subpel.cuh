@@ -27,6 +27,7 @@ struct IntParams {
   int g_lo, g_hi; // interior 16-column groups [g_lo, g_hi): every source word in-frame and aligned
   int border_bx;  // border blocks: groups per block row (power of two >= number of border groups)
   uint32_t k_hi;  // = kAvgHi (vavg4)
+  int vec_ok;     // W % 4 == 0 and rf 4-byte aligned: tile rows as aligned words (int_tile_kernel)
 };
 
 // Two columns per 32-bit register, one per 16-bit lane, and every lane kept
@@ -61,24 +62,9 @@ __device__ __forceinline__ uint32_t bytes_of(uint32_t a, uint32_t b) { return __
 // block, blockIdx.x = which border_bx-wide slice of the border groups (every
 // border group is covered: all of them when W % 4 != 0 or the RF rows are not
 // 4-byte aligned; dispatched first: they are the latency-bound tail otherwise).
-template <bool INTERIOR>
-__device__ __forceinline__ void int_body(const IntParams& P, int g, int rr) {
-  const int x0 = 16 * g - P.pad, y = rr - P.pad;
-
-  // source rows y-2 .. y+3 (k = 0..5), columns x0-4 .. x0+19 (c = 0..23, 6 words)
-  uint32_t w[6][6];
-#pragma unroll
-  for (int k = 0; k < 6; ++k) {
-    const int yy = clampi(y - 2 + k, 0, P.H - 1);
-    if (INTERIOR) {
-      const uint32_t* src = reinterpret_cast<const uint32_t*>(P.rf + (size_t)yy * P.W + x0 - 4);
-#pragma unroll
-      for (int q = 0; q < 6; ++q) w[k][q] = __ldg(src + q);
-    } else {
-#pragma unroll
-      for (int q = 0; q < 6; ++q) w[k][q] = load4_clamped(P.rf, P.W, P.H, x0 - 4 + 4 * q, yy);
-    }
-  }
+// the 16 planes of 16 columns x 1 row (plane group g, plane row rr) from the source words
+// w[k][q] = rows y-2 .. y+3 (k = 0..5), columns x0-4 .. x0+19 (q = 0..5), y = rr - pad, x0 = 16g - pad
+__device__ __forceinline__ void int_compute(const IntParams& P, int g, int rr, const uint32_t (&w)[6][6]) {
   // byte pairs as u16x2: pr[k][j] = columns (2j, 2j+1)
   auto pr = [&](int k, int j) -> uint32_t { return __byte_perm(w[k][j >> 1], 0, (j & 1) ? 0x4342 : 0x4140); };
 
@@ -180,6 +166,26 @@ __device__ __forceinline__ void int_body(const IntParams& P, int g, int rr) {
 #undef R_
 }
 
+template <bool INTERIOR>
+__device__ __forceinline__ void int_body(const IntParams& P, int g, int rr) {
+  const int x0 = 16 * g - P.pad, y = rr - P.pad;
+  // source rows y-2 .. y+3 (k = 0..5), columns x0-4 .. x0+19 (c = 0..23, 6 words)
+  uint32_t w[6][6];
+#pragma unroll
+  for (int k = 0; k < 6; ++k) {
+    const int yy = clampi(y - 2 + k, 0, P.H - 1);
+    if (INTERIOR) {
+      const uint32_t* src = reinterpret_cast<const uint32_t*>(P.rf + (size_t)yy * P.W + x0 - 4);
+#pragma unroll
+      for (int q = 0; q < 6; ++q) w[k][q] = __ldg(src + q);
+    } else {
+#pragma unroll
+      for (int q = 0; q < 6; ++q) w[k][q] = load4_clamped(P.rf, P.W, P.H, x0 - 4 + 4 * q, yy);
+    }
+  }
+  int_compute(P, g, rr, w);
+}
+
 #ifndef FEVES_INT_MINB
 #define FEVES_INT_MINB 1
 #endif
@@ -197,6 +203,69 @@ __global__ void __launch_bounds__(128, FEVES_INT_MINB) int_subpel_kernel(const I
     const int g = tb < P.g_lo ? tb : P.g_hi + (tb - P.g_lo);
     const int rr = P.row_begin + blockIdx.y * by + tr;
     if (rr < P.row_end) int_body<false>(P, g, rr);
+  }
+}
+
+// Shared-memory tiled INT: CTA = kIntTx plane groups (16 columns each) x kIntTy plane rows.
+// The source tile (kIntTy + 5 rows x 16 kIntTx + 8 columns, clamped, G5) is staged once with
+// coalesced 4-byte loads (each source word is read by 6 rows x 1.5 groups in the per-thread
+// kernel), then every thread reads its 6 x 6 words with LDS.128 + LDS.64 (its window starts
+// 16-byte aligned in the tile, so a warp's quarter-requests are bank-conflict free).
+constexpr int kIntTx = 8, kIntTy = 16;
+constexpr int kIntSrcRows = kIntTy + 5, kIntSrcWords = 4 * kIntTx + 2, kIntStride = 36;   // words per tile row
+static_assert(kIntStride >= kIntSrcWords && kIntStride % 4 == 0, "INT tile row stride");
+
+#ifndef FEVES_INT_TPC
+#define FEVES_INT_TPC 1   // tile rows per CTA (> 1: the next tile is copied while one computes; measured slower: 1 wave)
+#endif
+__device__ __forceinline__ void int_cp4(uint32_t* dst, const void* src) {
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"((uint32_t)__cvta_generic_to_shared(dst)), "l"(src));
+}
+
+__global__ void __launch_bounds__(kIntTx * kIntTy) int_tile_kernel(const IntParams P) {
+  __shared__ __align__(16) uint32_t tile[2][kIntSrcRows * kIntStride];
+  const int groups = P.pitch / 16;
+  const int g0 = kIntTx * blockIdx.x;
+  const int xs = 16 * g0 - P.pad - 4;                      // frame column of tile word 0
+  const int tid = threadIdx.y * kIntTx + threadIdx.x;
+  const bool fast = P.vec_ok && xs >= 0 && xs + 4 * kIntSrcWords <= P.W;
+  // stage the source tile of tile row ty (plane rows r0 .. r0+15) into buffer b
+  auto stage = [&](int ty, int b) {
+    const int ys = P.row_begin + kIntTy * ty - P.pad - 2;
+    for (int i = tid; i < kIntSrcRows * kIntSrcWords; i += kIntTx * kIntTy) {
+      const int r = i / kIntSrcWords, q = i - r * kIntSrcWords;
+      const int yy = clampi(ys + r, 0, P.H - 1);
+      uint32_t* d = &tile[b][r * kIntStride + q];
+      if (fast) int_cp4(d, reinterpret_cast<const uint32_t*>(P.rf + (size_t)yy * P.W + xs) + q);
+      else *d = load4_clamped(P.rf, P.W, P.H, xs + 4 * q, yy);
+    }
+    asm volatile("cp.async.commit_group;" ::: "memory");
+  };
+  const int n_ty = (P.row_end - P.row_begin + kIntTy - 1) / kIntTy;
+  const int ty0 = FEVES_INT_TPC * blockIdx.y, ty1 = min(n_ty, ty0 + FEVES_INT_TPC);
+  stage(ty0, 0);
+  for (int ty = ty0; ty < ty1; ++ty) {
+    const int b = (ty - ty0) & 1;
+    if (ty + 1 < ty1) {
+      stage(ty + 1, b ^ 1);                                  // in flight during this tile's compute
+      asm volatile("cp.async.wait_group 1;" ::: "memory");
+    } else {
+      asm volatile("cp.async.wait_group 0;" ::: "memory");
+    }
+    __syncthreads();
+    const int g = g0 + threadIdx.x, rr = P.row_begin + kIntTy * ty + threadIdx.y;
+    if (g < groups && rr < P.row_end) {
+      uint32_t w[6][6];
+#pragma unroll
+      for (int k = 0; k < 6; ++k) {
+        const uint32_t* t = tile[b] + (threadIdx.y + k) * kIntStride + 4 * threadIdx.x;
+        const uint4 a4 = *reinterpret_cast<const uint4*>(t);
+        const uint2 b2 = *reinterpret_cast<const uint2*>(t + 4);
+        w[k][0] = a4.x; w[k][1] = a4.y; w[k][2] = a4.z; w[k][3] = a4.w; w[k][4] = b2.x; w[k][5] = b2.y;
+      }
+      int_compute(P, g, rr, w);
+    }
+    __syncthreads();                                         // buffer b is restaged two tiles later
   }
 }
 

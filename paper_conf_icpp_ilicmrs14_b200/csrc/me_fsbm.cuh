@@ -37,11 +37,7 @@ namespace feves {
 #ifndef FEVES_ME_MINB
 #define FEVES_ME_MINB 4
 #endif
-#ifndef FEVES_ME_CUNROLL
-#define FEVES_ME_CUNROLL 1
-#endif
 constexpr int kMeT = FEVES_ME_T;   // candidates per vertical step
-constexpr int kMeCUnroll = FEVES_ME_CUNROLL;   // chunks per iteration of the dy sweep
 
 struct MeParams {
   const uint8_t* cf;
@@ -482,10 +478,7 @@ __global__ void __launch_bounds__(S_CT ? 128 : 256, S_CT ? FEVES_ME_MINB : 2) me
     }
     __syncthreads();
 
-    const int n_chunks = (S_CT ? me_dyl(S_CT) : DYL) / NSTG / kMeT;   // compile-time for S_CT > 0
-    // one chunk = kMeT candidates (dy0 .. dy0+kMeT-1) of this lane's dx column
-    auto chunk = [&](const int ci) __attribute__((always_inline)) {
-      const int c = hs * (DYL / NSTG) + ci * kMeT;
+    for (int c = hs * (DYL / NSTG); c < (hs + 1) * (DYL / NSTG); c += kMeT) {
       const int dy0 = min(dy_begin + c, hi + 1 - kMeT);   // clamped chunk: duplicates are harmless
       uint32_t rank[kMeT];
 #pragma unroll
@@ -544,15 +537,7 @@ __global__ void __launch_bounds__(S_CT ? 128 : 256, S_CT ? FEVES_ME_MINB : 2) me
           }
         }
       }
-    };
-    // kMeCUnroll chunks per iteration, so the compiler can overlap one chunk's key / fold
-    // tail (rows kMeT-1 .. kMeT+14, few VABSDIFF4) with the next chunk's head
-#pragma unroll 1
-    for (int ci = 0; ci + kMeCUnroll <= n_chunks; ci += kMeCUnroll) {
-#pragma unroll
-      for (int u = 0; u < kMeCUnroll; ++u) chunk(ci + u);
     }
-    for (int ci = n_chunks - n_chunks % kMeCUnroll; ci < n_chunks; ++ci) chunk(ci);
 
     if (QUAD && hs == 0) {                                // end of the dy < 0 quadrant half
 #pragma unroll

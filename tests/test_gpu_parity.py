@@ -556,3 +556,20 @@ def test_sme_staged_kernel_equals_oracle(feves, orc, lam, S, kind):
     np.testing.assert_array_equal(q.cpu().numpy().reshape(n, n_rf, 41, 2), o_q)
     np.testing.assert_array_equal(qs.cpu().numpy().reshape(n, n_rf, 41), o_qs)
     me.close()
+
+
+@pytest.mark.parametrize("W,H,S", [(64, 48, 8), (72, 52, 16), (854, 40, 32), (330, 170, 64), (33, 17, 128)])
+def test_int_kernels_equal_oracle(feves, orc, W, H, S):
+    """both INT kernels (ME_OPT_INT_KERNEL 0: per-thread global loads, 1: shared-memory tiles)
+    write every byte of the 16 planes == oracle, incl. ragged tiles and W % 4 != 0"""
+    rf = gen_noise(W, H, 0, W * H + S)
+    me = feves.MotionEstimator(W, H, S, 1)
+    ref = orc.int_planes(rf, me.sf_pad, me.sf_pitch, me.sf_rows)
+    for k in (0, 1):
+        me.set_option(me.OPT_INT_KERNEL, k)
+        sf = me.new_sf()
+        sf.fill_(0x5A)
+        me.interpolate(_dev(rf), out=sf)
+        torch.cuda.synchronize()
+        np.testing.assert_array_equal(sf.cpu().numpy(), ref, err_msg=f"int_kernel={k}")
+    me.close()
