@@ -416,6 +416,12 @@ def run_feves(args, cfg):
         dist.barrier()
     total_ms = float(tot.item())
     fps = args.steps / (total_ms / 1e3)
+    per_rank = None
+    if peer:                                         # each rank's device time per push (CUDA events)
+        ms = ss.stripe_ms()[-args.steps:]
+        mine = {"rank": rank, "rows": list(stripes(me.mb_rows, world)[rank]), "stripe_ms_mean": statistics.mean(ms)}
+        per_rank = [None] * world
+        dist.all_gather_object(per_rank, mine)
     mod_ms, mod, _ = timed(max(5, min(args.steps, 20)), True)
     graph_ab = None
     if world == 1:                                   # the other ME_OPT_GRAPH setting, same protocol
@@ -539,8 +545,8 @@ def run_feves(args, cfg):
                "h2d_bytes_per_step": pinned[0].numel(),
                "d2h_bytes_per_step": qm_h.numel() * 2 + qs_h.numel() * 2,
                "api": ("PeerStream.push (rank 0 uploads the pinned frame; each rank pulls its stripe + halo "
-                       "rows over peer memory and its SME stores into rank 0's buffer; two 4-byte NCCL "
-                       "all-reduces per frame)" if peer else
+                       "rows over peer memory on its copy-in stream, overlapping its previous frame, and its SME "
+                       "stores into rank 0's buffer; stream-ordered peer flags, no collective)" if peer else
                        "ShardedStream.push (NCCL broadcast in, per-rank me_stream_push, NCCL gather out)")
                       + ", pinned buffers on rank 0"}
     if not args.no_e2e and world == 1:
@@ -591,6 +597,7 @@ def run_feves(args, cfg):
                            "; INT runs concurrently with ME (P:86) on a side stream")},
         "clocks": ck,
         "graph_ab": graph_ab,
+        "per_rank": per_rank,
         "e2e": e2e,
         "gpu_launches": launches,
         "roofline": {"bound": "alu", "kernel": "me_fsbm_kernel<64,fused>" if fused else "me_fsbm_kernel<64>",

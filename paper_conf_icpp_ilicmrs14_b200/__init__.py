@@ -59,6 +59,10 @@ def lib():
         L.me_stream_push.argtypes = [P, P, i, P, P, i, P]
         L.me_stream_outputs.argtypes = [P, P, P]
         L.me_stream_join.argtypes = [P]
+        u32 = ctypes.c_uint32
+        L.me_stream_push_flags.argtypes = [P, P, i, P, P, i, P, P, u32, P, u32]
+        L.me_stream_wait_value.argtypes = [P, P, u32]
+        L.me_stream_write_value.argtypes = [P, P, u32]
         L.me_sync.argtypes = [P]
         L.me_set_timing.argtypes = [P, i]
         L.me_get_timings.argtypes = [P, P, P, P]
@@ -70,7 +74,8 @@ def lib():
         L.me_ipc_close.argtypes = [P, P]
         for fn in ("me_set_stream", "me_set_rows", "me_get_layout", "me_estimate", "int_interpolate",
                    "sme_refine", "me_encode_frame", "me_last_launch_count", "me_stream_reset",
-                   "me_stream_push", "me_stream_outputs", "me_stream_join", "me_sync", "me_set_timing", "me_get_timings", "me_set_fused", "me_set_option", "me_mode_decision",
+                   "me_stream_push", "me_stream_outputs", "me_stream_join", "me_sync", "me_stream_push_flags",
+                   "me_stream_wait_value", "me_stream_write_value", "me_set_timing", "me_get_timings", "me_set_fused", "me_set_option", "me_mode_decision",
                    "me_ipc_export", "me_ipc_open", "me_ipc_close"):
             getattr(L, fn).restype = i
         _lib = L
@@ -258,6 +263,18 @@ class MotionEstimator:
         _check(lib().me_stream_push(self._ctx, cf_ptr, 0, qmvs_ptr, qsads_ptr, 0, ctypes.byref(n)))
         return n.value
 
+    def stream_push_flags(self, cf_ptr: int, qmvs_ptr: int, qsads_ptr: int, wait_flag: int = 0, wait_value: int = 0,
+                          signal_flag: int = 0, signal_value: int = 0, bind_stream=True):
+        """me_stream_push_flags on raw device addresses: the frame pull waits for
+        *wait_flag >= wait_value on the copy-in stream, *signal_flag = signal_value once the
+        outputs are complete (addresses 0 = none).  Returns n_ref_used."""
+        n = ctypes.c_int()
+        if bind_stream:
+            self._bind_stream()
+        _check(lib().me_stream_push_flags(self._ctx, cf_ptr, 0, qmvs_ptr, qsads_ptr, 0, ctypes.byref(n),
+                                          wait_flag or None, wait_value, signal_flag or None, signal_value))
+        return n.value
+
     def sync(self):
         _check(lib().me_sync(self._ctx))
 
@@ -344,4 +361,15 @@ class MotionEstimator:
         return tuple(x.value for x in v)
 
 
-__all__ = ["MotionEstimator", "FevesError", "lib", "LIB_PATH", "N_PART", "N_PHASE"]
+def stream_wait_value(stream, flag_ptr: int, value: int):
+    """enqueue on a torch stream: wait until the 32-bit device word at flag_ptr >= value"""
+    _check(lib().me_stream_wait_value(ctypes.c_void_p(stream.cuda_stream), flag_ptr, value))
+
+
+def stream_write_value(stream, flag_ptr: int, value: int):
+    """enqueue on a torch stream: write value to the 32-bit device word at flag_ptr"""
+    _check(lib().me_stream_write_value(ctypes.c_void_p(stream.cuda_stream), flag_ptr, value))
+
+
+__all__ = ["MotionEstimator", "FevesError", "lib", "LIB_PATH", "N_PART", "N_PHASE", "stream_wait_value",
+           "stream_write_value"]

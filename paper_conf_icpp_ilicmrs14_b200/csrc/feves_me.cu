@@ -97,6 +97,9 @@ struct me_ctx {
   int graph;             // ME_OPT_GRAPH
   int sme_kernel;        // ME_OPT_SME_KERNEL: 0 global-load SME (default), 1 shared-memory staged
   int int_kernel;        // ME_OPT_INT_KERNEL: 0 per-thread global loads, 1 shared-memory tiled
+  // me_stream_push_flags: stream-ordered peer flags of the push being enqueued
+  const uint32_t* wait_flag; uint32_t wait_value;     // the frame copy waits for *wait_flag >= wait_value
+  uint32_t* signal_flag; uint32_t signal_value;       // written once the push's outputs are complete
   int* d_ovf;            // staged SME overflow list: [0] count, then (MB, RF) items
   bool capturing;        // push_enqueue runs inside a stream capture
   long long gepoch;      // bumped by every setting change: cached graphs are stale
@@ -146,6 +149,36 @@ static void graphs_drop(me_ctx* c) {
     if (g.graph) cudaGraphDestroy(g.graph);
   }
   c->graphs.clear();
+}
+
+// Stream memory operations (driver API, through cudaGetDriverEntryPoint like alloc_base):
+// a stream waits until a 32-bit device word (local or a peer's, me_ipc_open) is >= value, or
+// writes one after its preceding work -- the stream-ordered flags of the multi-GPU exchange.
+using StreamValueFn = CUresult (*)(CUstream, CUdeviceptr, cuuint32_t, unsigned int);
+static StreamValueFn driver_fn(const char* name) {
+  void* f = nullptr;
+  cudaDriverEntryPointQueryResult q;
+  if (cudaGetDriverEntryPoint(name, &f, cudaEnableDefault, &q) != cudaSuccess || !f || q != cudaDriverEntryPointSuccess) {
+    cudaGetLastError();
+    return nullptr;
+  }
+  return reinterpret_cast<StreamValueFn>(f);
+}
+static int stream_wait_value(cudaStream_t s, const uint32_t* flag, uint32_t value) {
+  static StreamValueFn fn = driver_fn("cuStreamWaitValue32");
+  if (!fn) return ME_ECUDA;
+  return fn(reinterpret_cast<CUstream>(s), reinterpret_cast<CUdeviceptr>(flag), value, CU_STREAM_WAIT_VALUE_GEQ) ==
+                 CUDA_SUCCESS
+             ? ME_OK
+             : ME_ECUDA;
+}
+static int stream_write_value(cudaStream_t s, uint32_t* flag, uint32_t value) {
+  static StreamValueFn fn = driver_fn("cuStreamWriteValue32");
+  if (!fn) return ME_ECUDA;
+  return fn(reinterpret_cast<CUstream>(s), reinterpret_cast<CUdeviceptr>(flag), value, CU_STREAM_WRITE_VALUE_DEFAULT) ==
+                 CUDA_SUCCESS
+             ? ME_OK
+             : ME_ECUDA;
 }
 
 static int launch_status() {
@@ -740,10 +773,14 @@ static int push_enqueue(me_ctx* c, const uint8_t* cf, int cf_on_host, int16_t* o
     if (c->fv0[s] > y0 || c->fv1[s] < y1) return ME_ESTATE;
   }
   const size_t off = (size_t)y0 * c->W, len = (size_t)(y1 - y0) * c->W;
-  if (cf_on_host) {
-    // upload on the copy-in stream once the compute of push t-2 (last reader of this slot) is done
-    if (cudaStreamWaitEvent(c->copy_in, c->ev_done[par], 0) != cudaSuccess ||
-        cudaMemcpyAsync(cur + off, cf + off, len, cudaMemcpyHostToDevice, c->copy_in) != cudaSuccess ||
+  if (cf_on_host || c->wait_flag) {
+    // upload (host frame) / pull (device or peer frame published with a flag) on the copy-in
+    // stream once the compute of push t-2 (last reader of this slot) is done, so it overlaps the
+    // compute of push t-1 (P:51 copy engines; SURVEY §8(e) frame t+1 under frame t's compute)
+    if (cudaStreamWaitEvent(c->copy_in, c->ev_done[par], 0) != cudaSuccess) return launch_status();
+    if (c->wait_flag && (st = stream_wait_value(c->copy_in, c->wait_flag, c->wait_value)) != ME_OK) return st;
+    if (cudaMemcpyAsync(cur + off, cf + off, len, cf_on_host ? cudaMemcpyHostToDevice : cudaMemcpyDefault,
+                        c->copy_in) != cudaSuccess ||
         cudaEventRecord(c->ev_up[par], c->copy_in) != cudaSuccess ||
         cudaStreamWaitEvent(c->stream, c->ev_up[par], 0) != cudaSuccess)
       return launch_status();
@@ -797,6 +834,9 @@ static int push_enqueue(me_ctx* c, const uint8_t* cf, int cf_on_host, int16_t* o
       if ((st = run_me_sme(c, cur, rfs, sfs, c->d_mvs, c->d_sads, qm, qs, n_ref, c->ev_join)) != ME_OK) return st;
     }
     const size_t nmv = (size_t)(c->row1 - c->row0) * c->mb_cols * c->n_rf * kNPart;
+    if (c->signal_flag && (st = stream_write_value(c->ov_pending ? c->ov_st : c->stream, c->signal_flag,
+                                                   c->signal_value)) != ME_OK)
+      return st;
     if (cudaEventRecord(c->ev_done[par], c->ov_pending ? c->ov_st : c->stream) != cudaSuccess) return launch_status();
     if (out_on_host) {   // download on the copy-out stream, overlapping the next frame's compute
       // only the n_ref searched RF slots of every MB (slots >= n_ref stay untouched, as for
@@ -811,8 +851,9 @@ static int push_enqueue(me_ctx* c, const uint8_t* cf, int cf_on_host, int16_t* o
           cudaEventRecord(c->ev_down[par], c->copy_out) != cudaSuccess)
         return launch_status();
     }
-  } else if (cudaEventRecord(c->ev_done[par], c->stream) != cudaSuccess) {
-    return launch_status();
+  } else {
+    if (c->signal_flag && (st = stream_write_value(c->stream, c->signal_flag, c->signal_value)) != ME_OK) return st;
+    if (cudaEventRecord(c->ev_done[par], c->stream) != cudaSuccess) return launch_status();
   }
   c->t = t + 1;
   return ME_OK;
@@ -852,6 +893,7 @@ extern "C" int me_stream_push(me_ctx* c, const uint8_t* cf, int cf_on_host, int1
   if (st != ME_OK) return st;
   const int period = graph_period(c);
   const bool graph = c->graph && !cf_on_host && !out_on_host && !c->overlap && !c->pipeline && !c->fuse &&
+                     !c->wait_flag && !c->signal_flag &&
                      c->t >= c->n_rf && period <= 64 && !push_needs_sf_refresh(c);
   if (!graph) return push_enqueue(c, cf, cf_on_host, out_qmvs, out_qsads, out_on_host, n_ref_used);
   return push_graph(c, cf, out_qmvs, out_qsads, n_ref_used, period);
@@ -945,6 +987,28 @@ static int push_graph(me_ctx* c, const uint8_t* cf, int16_t* out_qmvs, uint16_t*
       cudaEventRecord(c->ev_done[par], c->stream) != cudaSuccess)   // a real record (the captured one is a node)
     return launch_status();
   return ME_OK;
+}
+
+extern "C" int me_stream_push_flags(me_ctx* c, const uint8_t* cf, int cf_on_host, int16_t* out_qmvs,
+                                    uint16_t* out_qsads, int out_on_host, int* n_ref_used, const uint32_t* wait_flag,
+                                    uint32_t wait_value, uint32_t* signal_flag, uint32_t signal_value) {
+  if (!c) return ME_EINVAL;
+  if ((wait_flag && !is_device_ptr(c, wait_flag)) || (signal_flag && !is_device_ptr(c, signal_flag))) return ME_EINVAL;
+  c->wait_flag = wait_flag; c->wait_value = wait_value;
+  c->signal_flag = signal_flag; c->signal_value = signal_value;
+  const int st = me_stream_push(c, cf, cf_on_host, out_qmvs, out_qsads, out_on_host, n_ref_used);
+  c->wait_flag = nullptr; c->signal_flag = nullptr;
+  return st;
+}
+
+extern "C" int me_stream_wait_value(void* stream, const uint32_t* flag, uint32_t value) {
+  if (!flag) return ME_EINVAL;
+  return stream_wait_value(reinterpret_cast<cudaStream_t>(stream), flag, value);
+}
+
+extern "C" int me_stream_write_value(void* stream, uint32_t* flag, uint32_t value) {
+  if (!flag) return ME_EINVAL;
+  return stream_write_value(reinterpret_cast<cudaStream_t>(stream), flag, value);
 }
 
 extern "C" int me_sync(me_ctx* c) {

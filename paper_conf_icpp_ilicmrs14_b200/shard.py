@@ -182,32 +182,38 @@ class ShardedStream:
 
 
 class PeerStream:
-    """IPPP stream over G ranks with the exchange done in peer memory (SURVEY §8(e),
-    "Option to fuse the collective"; BJ north_star "reference-frame rows plus an
-    SA-radius halo via ... P2P over NVLink").
+    """IPPP stream over G ranks with the exchange done in peer memory and ordered by
+    stream-ordered flags ("Option to fuse the collective"; BJ north_star
+    "reference-frame rows plus an SA-radius halo via ... P2P over NVLink"; P:51 / P:89: the
+    transfers overlap the computation).  No collective and no host synchronisation per frame.
 
-    Rank ``src`` owns two frame slots and two full-frame output buffers and exports
-    them (``me_ipc_export``); every other rank maps them (``me_ipc_open``).  Per frame t:
-      1. rank src copies frame t into slot t mod 2;
-      2. barrier #1 (stream-ordered: a 4-byte NCCL all-reduce, no host sync);
-      3. every rank runs ``me_stream_push`` with the frame read from rank src's slot
-         (``ME_OPT_HALO_ONLY``: the copy engine pulls only the stripe + halo rows,
-         [16 r0 - R - 6, 16 r1 + R + 7), over NVLink) and with the outputs pointed at
-         its stripe's rows of rank src's output buffer t mod 2: the SME kernel's
-         stores travel over NVLink, so there is no gather collective and no copy;
-      4. barrier #2: every stripe of frame t is in rank src's buffer.
-    Slot reuse is safe: rank src overwrites slot t mod 2 at frame t+2, after barrier
-    #2 of frame t+1, which every rank passes only after its push of frame t has read
-    that slot.  The tensors returned on rank src stay valid until push t+2.
-    Results equal the single-GPU stream bitwise (pin P11); the split is the static
-    equidistant one -- with the adaptive re-split use ``ShardedStream``.
-    Over gloo (one shared GPU in tests) the barriers synchronise the host instead."""
+    Rank ``src`` owns two frame slots, two full-frame output buffers and a done-flag word per
+    rank; every rank owns two ready-flag words.  All are exported (``me_ipc_export``) and
+    mapped by the others (``me_ipc_open``).  Flags are only ever WAITED on locally and
+    WRITTEN remotely (``me_stream_wait_value`` / ``me_stream_write_value``).  Per frame t:
+      rank src, publish stream:  wait for the start of its push t-1 (so everything up to the
+          consumer of frame t-2 and the waits for its done flags have run), copy frame t into
+          slot t mod 2, write ready[t mod 2] = t+1 into every rank's flag words;
+      every rank, its stream:    ``me_stream_push_flags``: the copy-in stream waits for its own
+          ready[t mod 2] >= t+1, pulls ONLY its stripe + halo rows from rank src's slot
+          (``ME_OPT_HALO_ONLY``, copy engine over NVLink) -- overlapping its compute of frame
+          t-1 --, runs INT || ME -> SME with the SME stores going straight into its stripe's rows
+          of rank src's output buffer t mod 2, then writes done[rank] = t+1 into rank src's
+          memory;
+      rank src, its stream:      waits for done[r] >= t+1 of every rank.
+    Slot / buffer reuse: slot and output buffer t mod 2 are rewritten at frame t+2, whose
+    ready flag is written only after rank src passed the done-waits of frame t and whatever its
+    caller enqueued after push t (e.g. the D2H of frame t's outputs).  The tensors returned on
+    rank src are complete in its stream order and stay valid until push t+2.  Results equal
+    the single-GPU stream bitwise (pin P11); the split is the static equidistant one.
+    ``stripe_ms()`` gives each push's device time on this rank (CUDA events)."""
 
     def __init__(self, me, group=None, src: int = 0):
+        import paper_conf_icpp_ilicmrs14_b200 as F
+        self.F = F
         self.me, self.group, self.src = me, group, src
         self.rank = dist.get_rank(group)
         self.world = dist.get_world_size(group)
-        self.nccl = dist.get_backend(group) == "nccl"
         self.cur = stripes(me.mb_rows, self.world)
         r0, r1 = self.cur[self.rank]
         me.set_rows(r0, r1)
@@ -216,53 +222,78 @@ class PeerStream:
         H, W = me.height, me.width
         shape = (me.mb_rows, me.mb_cols, me.n_rf, 41)
         self.row_bytes = (me.mb_cols * me.n_rf * 41 * 4, me.mb_cols * me.n_rf * 41 * 2)
+        self.ready = torch.zeros(2, dtype=torch.int32, device=dev)              # mine: waited on locally
+        mine = [me.ipc_export(self.ready) + (8,)]
         if self.rank == src:
             self.frames = [torch.empty((H, W), dtype=torch.uint8, device=dev) for _ in range(2)]
             self.qm = [torch.empty(shape + (2,), dtype=torch.int16, device=dev) for _ in range(2)]
             self.qs = [torch.empty(shape, dtype=torch.uint16, device=dev) for _ in range(2)]
-            bufs = self.frames + self.qm + self.qs
-            exported = [me.ipc_export(b) + (b.numel() * b.element_size(),) for b in bufs]
-        else:
-            exported = None
+            self.done = torch.zeros(self.world, dtype=torch.int32, device=dev)
+            bufs = self.frames + self.qm + self.qs + [self.done]
+            mine += [me.ipc_export(b) + (b.numel() * b.element_size(),) for b in bufs]
         allx = [None] * self.world
-        dist.all_gather_object(allx, exported, group=group)
+        dist.all_gather_object(allx, mine, group=group)
+        self.opened = []
+
+        def open_(h):
+            p = me.ipc_open(*h)
+            self.opened.append(p)
+            return p
         if self.rank == src:
             ptrs = [b.data_ptr() for b in bufs]
-            self.opened = []
+            # every rank's ready words (own: local address)
+            self.ready_ptrs = [self.ready.data_ptr() if r == src else open_(allx[r][0]) for r in range(self.world)]
+            self.pub = torch.cuda.Stream(device=dev)
+            self.ev_start = [torch.cuda.Event(), torch.cuda.Event()]
         else:
-            ptrs = [me.ipc_open(h, off, n) for h, off, n in allx[src]]
-            self.opened = list(ptrs)
+            ptrs = [open_(h) for h in allx[src][1:]]
         self.f_ptr, self.qm_ptr, self.qs_ptr = ptrs[0:2], ptrs[2:4], ptrs[4:6]
-        self.flag = torch.zeros(1, dtype=torch.int32, device=dev if self.nccl else "cpu")
+        self.done_ptr = ptrs[6]                                              # rank src's done words
         self.t = 0
-
-    def _barrier(self):
-        if self.nccl:
-            dist.all_reduce(self.flag, group=self.group)   # ordered on the current stream
-        else:
-            torch.cuda.current_stream(self.me.device).synchronize()
-            dist.barrier(group=self.group)
+        self.times = []
+        dist.barrier(group=group)
 
     def push(self, frame, frame_buf=None):
         """frame: this step's frame on rank ``src`` (device or pinned host tensor [H, W]);
-        ignored elsewhere.  Returns (qmvs, qsads, n_ref) of the WHOLE frame on rank src,
-        None elsewhere."""
-        b = self.t & 1
+        ignored elsewhere.  Returns (qmvs, qsads, n_ref) of the WHOLE frame on rank src
+        (complete in its stream order), None elsewhere."""
+        F, t, b = self.F, self.t, self.t & 1
+        cs = torch.cuda.current_stream(self.me.device)
         if self.rank == self.src:
-            self.frames[b].copy_(frame.view(self.me.height, self.me.width), non_blocking=True)
-        self._barrier()
+            self.ev_start[b].record(cs)
+            with torch.cuda.stream(self.pub):
+                if t >= 1:
+                    self.pub.wait_event(self.ev_start[b ^ 1])               # start of push t-1
+                self.frames[b].copy_(frame.view(self.me.height, self.me.width), non_blocking=True)
+                for p in self.ready_ptrs:
+                    F.stream_write_value(self.pub, p + 4 * b, t + 1)
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(cs)
         r0 = self.cur[self.rank][0]
-        n_ref = self.me.stream_push_ptr(self.f_ptr[b], self.qm_ptr[b] + r0 * self.row_bytes[0],
-                                        self.qs_ptr[b] + r0 * self.row_bytes[1])
-        self._barrier()
+        n_ref = self.me.stream_push_flags(self.f_ptr[b], self.qm_ptr[b] + r0 * self.row_bytes[0],
+                                          self.qs_ptr[b] + r0 * self.row_bytes[1],
+                                          wait_flag=self.ready.data_ptr() + 4 * b, wait_value=t + 1,
+                                          signal_flag=self.done_ptr + 4 * self.rank, signal_value=t + 1)
+        e1.record(cs)
+        self.times.append((e0, e1))
         self.t += 1
         if self.rank == self.src:
+            for r in range(self.world):
+                F.stream_wait_value(cs, self.done_ptr + 4 * r, t + 1)
             return self.qm[b], self.qs[b], n_ref
         return None
 
+    def stripe_ms(self):
+        """device time of each push on this rank (ms; CUDA events on its stream, P:87 / P:218)"""
+        torch.cuda.synchronize(self.me.device)
+        return [a.elapsed_time(b) for a, b in self.times]
+
     def close(self):
-        """Unmap rank src's buffers (collective: rank src keeps them alive until all closed)."""
+        """Unmap the peer buffers (collective: every rank keeps its exported memory alive until
+        all have unmapped)."""
         self.me.sync()
+        torch.cuda.synchronize(self.me.device)
+        dist.barrier(group=self.group)
         for p in self.opened:
             self.me.ipc_close(p)
         self.opened = []
