@@ -97,7 +97,6 @@ struct me_ctx {
   int graph;             // ME_OPT_GRAPH
   int sme_kernel;        // ME_OPT_SME_KERNEL: 0 global-load SME (default), 1 shared-memory staged
   int int_kernel;        // ME_OPT_INT_KERNEL: 0 per-thread global loads, 1 shared-memory tiled
-  int me_kernel;         // ME_OPT_ME_KERNEL: 0 one CTA per MB, 1 persistent with window prefetch (S 16/32/64)
   // me_stream_push_flags: stream-ordered peer flags of the push being enqueued
   const uint32_t* wait_flag; uint32_t wait_value;     // the frame copy waits for *wait_flag >= wait_value
   uint32_t* signal_flag; uint32_t signal_value;       // written once the push's outputs are complete
@@ -456,7 +455,6 @@ static int launch_me(me_ctx* c, const uint8_t* cf, const uint8_t* const* rfs, in
   bool vec = (c->W % 16 == 0) && (c->R % 16 == 0);
   for (int k = 0; k < n_ref; ++k) vec = vec && ((reinterpret_cast<uintptr_t>(rfs[k]) & 15) == 0);
   P.vec_ok = vec ? 1 : 0;
-  P.cf_vec16 = (c->W % 16 == 0) && ((reinterpret_cast<uintptr_t>(cf) & 15) == 0);
   const bool fused = sfs != nullptr;
   if (fused) {
     for (int k = 0; k < n_ref; ++k) P.sf[k] = sfs[k];
@@ -470,10 +468,9 @@ static int launch_me(me_ctx* c, const uint8_t* cf, const uint8_t* const* rfs, in
   if (c->me_ctas_per_sm > 0)   // occupancy cap: leave registers / warps for a co-running SME
     smem = std::max(smem, (size_t)(228 * 1024) / (size_t)(c->me_ctas_per_sm + 1) - 1024 + 64);
   tmark(c, 2, st);
-  const bool pf_ok = c->me_kernel == 1 && !c->inclusive && mvs && sads && (c->S == 16 || c->S == 32 || c->S == 64);
   const int variant = fused ? kMeFused
                     : c->max_pmv ? (c->lambda ? kMePmvRate : kMePmv)
-                    : c->lambda ? kMeRate : pf_ok ? kMePf : kMePlain;
+                    : c->lambda ? kMeRate : kMePlain;
   cudaError_t e;
   switch (c->inclusive || (c->max_pmv && c->S == 128) ? 0 : c->S) {   // compile-time window geometry for the paper's SA sizes (Fig. 6a: 32..256)
     case 16: e = me_launch_16(variant, grid, c->me_threads, smem, st, P); break;
@@ -1076,10 +1073,6 @@ extern "C" int me_set_option(me_ctx* c, int option, int value) {
   c->gepoch++;                                          // cached stream graphs are stale
   switch (option) {
     case ME_OPT_GRAPH: c->graph = value ? 1 : 0; return ME_OK;
-    case ME_OPT_ME_KERNEL:
-      if (value < 0 || value > 1) return ME_EINVAL;
-      c->me_kernel = value;
-      return ME_OK;
     case ME_OPT_INT_KERNEL:
       if (value < 0 || value > 1) return ME_EINVAL;
       c->int_kernel = value;

@@ -4,7 +4,6 @@
 #pragma once
 #include <algorithm>
 #include "me_fsbm.cuh"
-#include "me_fsbm_pf.cuh"
 #include "sme_refine.cuh"
 
 namespace feves {
@@ -16,7 +15,6 @@ enum MeVariant : int {
   kMeRate = 2,      // J = SAD + lambda * R (G18), key shift 15
   kMePmv = 3,       // predicted-MV centre (G21)
   kMePmvRate = 4,   // both
-  kMePf = 5,        // pure SAD, persistent with the next window prefetched (me_fsbm_pf.cuh; S = 16/32/64)
 };
 
 template <int SS>
@@ -31,22 +29,6 @@ inline cudaError_t me_launch_tmpl(int variant, dim3 grid, int threads, size_t sm
     case kMePmvRate:
       if constexpr (SS != 128) { me_fsbm_kernel<SS, false, 15, true><<<grid, threads, smem, st>>>(P); break; }
       return cudaErrorInvalidValue;
-    case kMePf:
-      if constexpr (SS == 16 || SS == 32 || SS == 64) {
-        static int per_sm = 0, n_sm = 0;
-        const size_t pf_smem = (size_t)me_pf_smem_words(SS) * 4;
-        if (!per_sm) {
-          int dev = 0;
-          cudaGetDevice(&dev);
-          cudaDeviceGetAttribute(&n_sm, cudaDevAttrMultiProcessorCount, dev);
-          cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, me_pf_kernel<SS>, threads, pf_smem);
-          if (per_sm < 1) per_sm = 1;
-        }
-        const int n_items = (int)(grid.x * grid.y);
-        me_pf_kernel<SS><<<std::min(n_items, per_sm * n_sm), threads, pf_smem, st>>>(P, n_items);
-        break;
-      }
-      return cudaErrorInvalidValue;
     default: me_fsbm_kernel<SS, false><<<grid, threads, smem, st>>>(P); break;
   }
   return cudaGetLastError();
@@ -57,10 +39,6 @@ inline cudaError_t me_set_smem_tmpl(int bytes) {
   cudaError_t e = cudaFuncSetAttribute(me_fsbm_kernel<SS>, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
   if (e == cudaSuccess) e = cudaFuncSetAttribute(me_fsbm_kernel<SS, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
   if (e == cudaSuccess) e = cudaFuncSetAttribute(me_fsbm_kernel<SS, false, 15>, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
-  if constexpr (SS == 16 || SS == 32 || SS == 64) {
-    if (e == cudaSuccess)
-      e = cudaFuncSetAttribute(me_pf_kernel<SS>, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
-  }
   if constexpr (SS != 128) {
     if (e == cudaSuccess)
       e = cudaFuncSetAttribute(me_fsbm_kernel<SS, false, 16, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);

@@ -56,7 +56,6 @@ struct MeParams {
   const int16_t* pmv;         // G21 predictor [frame MB][rf_stride][2] integer-pel (runtime-S kernel only), or null
   int max_pmv;                // G21 clamp of each predictor component
   int vec_ok;                 // 16-byte aligned rows and window start: vector staging allowed
-  int cf_vec16;               // W % 16 == 0 and cf 16-byte aligned (me_pf_kernel: CF rows by cp.async)
   // fused SME (template FUSE): SF of each RF, quarter-pel outputs
   const uint8_t* sf[kMaxRf];
   int sf_pad, sf_pitch;

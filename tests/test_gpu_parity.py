@@ -573,30 +573,3 @@ def test_int_kernels_equal_oracle(feves, orc, W, H, S):
         torch.cuda.synchronize()
         np.testing.assert_array_equal(sf.cpu().numpy(), ref, err_msg=f"int_kernel={k}")
     me.close()
-
-
-@pytest.mark.parametrize("W,H,S,n_rf,kind", [(64, 48, 16, 2, "tex"), (72, 52, 32, 3, "noise"), (96, 80, 64, 2, "flat"),
-                                             (200, 72, 32, 1, "tex"), (33, 17, 16, 1, "noise"), (150, 90, 64, 4, "tex")])
-def test_me_prefetch_kernel_equals_oracle(feves, orc, W, H, S, n_rf, kind):
-    """ME_OPT_ME_KERNEL = 1: the persistent ME kernel with the next (MB, RF) window prefetched by
-    cp.async (both buffers alternating per window of the CTA, ragged and unaligned frames through
-    the clamped path) == oracle, every MB; then the stream path on it"""
-    cf, rfs = _frames(kind, W, H, n_rf, 300 + W + S)
-    me = feves.MotionEstimator(W, H, S, n_rf)
-    me.set_option(me.OPT_ME_KERNEL, 1)
-    mvs, sads = me.estimate(_dev(cf), [_dev(r) for r in rfs])
-    torch.cuda.synchronize()
-    n = me.mb_rows * me.mb_cols
-    o_m, o_s = orc.me(cf, rfs, S)
-    np.testing.assert_array_equal(sads.cpu().numpy().reshape(n, n_rf, 41), o_s)
-    np.testing.assert_array_equal(mvs.cpu().numpy().reshape(n, n_rf, 41, 2), o_m)
-    frames = [gen_tex(W, H, t, 7 + S) for t in range(n_rf + 2)]
-    for t, f in enumerate(frames):
-        qm, qs, used = me.stream_push(_dev(f))
-    torch.cuda.synchronize()
-    rr = [frames[-2 - k] for k in range(n_rf)]
-    o_m2, _ = orc.me(frames[-1], rr, S)
-    o_q, o_qs = orc.sme(frames[-1], rr, o_m2)
-    np.testing.assert_array_equal(qm.cpu().numpy().reshape(n, n_rf, 41, 2), o_q)
-    np.testing.assert_array_equal(qs.cpu().numpy().reshape(n, n_rf, 41), o_qs)
-    me.close()
