@@ -133,6 +133,29 @@ __device__ __forceinline__ uint32_t sf_ld(const uint32_t* p) {
 #endif
 }
 struct Win2 { uint32_t l, r; };
+#ifndef FEVES_SME_OFF32
+#define FEVES_SME_OFF32 1
+#endif
+#if FEVES_SME_OFF32
+// a sweep's row pointer as a 32-bit word offset from ONE shared 64-bit base (the SF's first
+// word): 2 registers per row pointer instead of 3 (the kernel is register-capped at 80)
+struct RowP { const uint32_t* w0; uint32_t o, sh; };
+__device__ __forceinline__ RowP rowp_at(const uint8_t* sf, size_t byte_off) {
+  const uintptr_t a = reinterpret_cast<uintptr_t>(sf);
+  const uint32_t b = (uint32_t)(a & 3) + (uint32_t)byte_off;
+  return {reinterpret_cast<const uint32_t*>(a & ~uintptr_t(3)), b >> 2, 8u * (b & 3)};
+}
+__device__ __forceinline__ Win2 ld_lr(const RowP& q, int off) {   // off = row * (pitch / 4)
+  const uint32_t* p = q.w0 + (q.o + (uint32_t)off);
+  const uint32_t w0 = sf_ld(p), w1 = sf_ld(p + 1);
+  return {__funnelshift_r(w0, w1, q.sh), __funnelshift_rc(w0, w1, q.sh + 8u)};
+}
+__device__ __forceinline__ uint32_t ld_w(const RowP& q, int off) {
+  const uint32_t* p = q.w0 + (q.o + (uint32_t)off);
+  return __funnelshift_r(sf_ld(p), sf_ld(p + 1), q.sh);
+}
+#define FEVES_ROWP(sf, p) rowp_at((sf), (size_t)((p) - (sf)))
+#else
 struct RowP { const uint32_t* w; uint32_t sh; };
 __device__ __forceinline__ RowP rowp(const uint8_t* p) {
   const uintptr_t a = reinterpret_cast<uintptr_t>(p);
@@ -145,6 +168,8 @@ __device__ __forceinline__ Win2 ld_lr(const RowP& q, int off) {   // off = row *
 __device__ __forceinline__ uint32_t ld_w(const RowP& q, int off) {
   return __funnelshift_r(sf_ld(q.w + off), sf_ld(q.w + off + 1), q.sh);
 }
+#define FEVES_ROWP(sf, p) rowp(p)
+#endif
 
 // Half stage, SAD, one block group of HR rows (DESIGN.md §6 "row sweep"): for the
 // full-pel centre (mx, my) the 8 ring candidates c + 2 s_k are windows of three
@@ -161,9 +186,9 @@ __device__ __forceinline__ void half_sad_sweep(const uint8_t* __restrict__ sf, s
                                                const uint8_t* base, int mx, int my, const uint32_t* cf,
                                                uint32_t (&sad)[8]) {
   // base = plane 0 at the strip's top-left integer sample (pad applied)
-  const RowP ph = rowp(base + 8 * plane + (ptrdiff_t)(my - 1) * pitch + mx);
-  const RowP pj = rowp(base + 10 * plane + (ptrdiff_t)(my - 1) * pitch + (mx - 1));
-  const RowP pb = rowp(base + 2 * plane + (ptrdiff_t)my * pitch + (mx - 1));
+  const RowP ph = FEVES_ROWP(sf, base + 8 * plane + (ptrdiff_t)(my - 1) * pitch + mx);
+  const RowP pj = FEVES_ROWP(sf, base + 10 * plane + (ptrdiff_t)(my - 1) * pitch + (mx - 1));
+  const RowP pb = FEVES_ROWP(sf, base + 2 * plane + (ptrdiff_t)my * pitch + (mx - 1));
   const int wp = pitch >> 2;
 #pragma unroll
   for (int k = 0; k < 8; ++k) sad[k] = 0;
@@ -202,17 +227,17 @@ __device__ __forceinline__ uint32_t quarter_win(const uint32_t (&hp)[3][3], int 
 // the sweep reads "outer" rows (hy+-1 parity) r = 0..HR and "middle" rows (hy
 // parity) r = 0..HR-1, 4 LDG each, and CF row r uses outer r, middle r, outer r+1.
 template <int HR>
-__device__ __forceinline__ void quarter_sad_sweep(size_t plane, int pitch, const uint8_t* base, int hx, int hy,
-                                                  const uint32_t* cf, uint32_t (&qs)[8], uint32_t kh) {
+__device__ __forceinline__ void quarter_sad_sweep(const uint8_t* sf, size_t plane, int pitch, const uint8_t* base,
+                                                  int hx, int hy, const uint32_t* cf, uint32_t (&qs)[8], uint32_t kh) {
   const bool mixed = ((hx ^ hy) & 1) != 0;
   const int xm = hx - 1, x0 = hx, ym = hy - 1, y0 = hy;
   auto at = [&](int X, int Y) {                 // plane row pointer of half-grid point (X, Y), CF row 0
     return base + (size_t)(8 * (Y & 1) + 2 * (X & 1)) * plane + (ptrdiff_t)(Y >> 1) * pitch + (X >> 1);
   };
-  const RowP o_lr = rowp(at(xm, ym));           // outer rows, columns hx-1 / hx+1
-  const RowP o_c = rowp(at(x0, ym));            // outer rows, column hx
-  const RowP m_lr = rowp(at(xm, y0));           // middle rows
-  const RowP m_c = rowp(at(x0, y0));
+  const RowP o_lr = FEVES_ROWP(sf, at(xm, ym));   // outer rows, columns hx-1 / hx+1
+  const RowP o_c = FEVES_ROWP(sf, at(x0, ym));    // outer rows, column hx
+  const RowP m_lr = FEVES_ROWP(sf, at(xm, y0));   // middle rows
+  const RowP m_c = FEVES_ROWP(sf, at(x0, y0));
   const int wp = pitch >> 2;
 #pragma unroll
   for (int k = 0; k < 8; ++k) qs[k] = 0;
@@ -344,7 +369,8 @@ __device__ __forceinline__ void refine_mode(const SmeParams& P, const uint8_t* _
       const int hx = bvx >> 1, hy = bvy >> 1;          // half-grid coordinates (bvx, bvy even)
       uint32_t qs[8];
       if (!SATD) {                                     // SAD: one row sweep
-        quarter_sad_sweep<4 * YG>(P.plane, P.pitch, sf + (size_t)(yg + P.pad) * P.pitch + (xs + P.pad), hx, hy, cf, qs, P.k_hi);
+        quarter_sad_sweep<4 * YG>(sf, P.plane, P.pitch, sf + (size_t)(yg + P.pad) * P.pitch + (xs + P.pad), hx, hy, cf, qs,
+                                  P.k_hi);
       } else {                                         // SATD: whole 4x4 blocks, one candidate at a time
         const bool mixed = ((hx ^ hy) & 1) != 0;
         int off[3][3];                                 // window offsets from the strip's row base
@@ -400,7 +426,7 @@ __device__ __forceinline__ void refine_mode(const SmeParams& P, const uint8_t* _
 }
 
 #ifndef FEVES_SME_MINB
-#define FEVES_SME_MINB 6   // 80 registers, 6 CTAs x 4 warps per SM (measured: 1 -> 243 regs 248 us; 6 -> 183 us; 8 -> 184 us; 10 -> 194 us)
+#define FEVES_SME_MINB 5   // 96 registers, 5 CTAs x 4 warps per SM; with 32-bit row offsets (FEVES_SME_OFF32) 8 B of stack, 1 spill + 3 reloads per partition group outside the sweeps (was 72 B / 56 sites at 80 registers); 4 (128 registers): none, 147.5 vs 145.4 us; 5 / 6: 145.4 us
 #endif
 template <bool RD, bool SATD>
 __global__ void __launch_bounds__(128, FEVES_SME_MINB) sme_refine_kernel(const SmeParams P) {
