@@ -226,9 +226,12 @@ class OracleSampler:
         t0 = time.perf_counter()
         mv, _ = orc.me(self.cf, self.rfs, cfg.sa_range, mb_list=mbs, threads=self.threads)
         t1 = time.perf_counter()
-        orc.sme(self.cf, self.rfs, mv, mb_list=mbs, threads=self.threads)
+        me_only = cfg.path == "me"                      # BASELINE configs 1-2: integer ME only
+        if not me_only:
+            orc.sme(self.cf, self.rfs, mv, mb_list=mbs, threads=self.threads)
         t2 = time.perf_counter()
-        orc.int_planes(self.rfs[0], pad, pitch, rows, row_begin=0, row_end=int_rows, threads=self.threads)
+        if not me_only:
+            orc.int_planes(self.rfs[0], pad, pitch, rows, row_begin=0, row_end=int_rows, threads=self.threads)
         t3 = time.perf_counter()
         t = t3 - t0
         fps = (min(n, self.n_total) / self.n_total) / t
@@ -236,6 +239,9 @@ class OracleSampler:
                 f"(the newest RF; stream mode)" if full else
                 f"{n} of {self.n_total} MBs (seeded) x {cfg.n_rf} RFs ME+SME and {int_rows} of {rows} SF rows of "
                 f"one INT, extrapolated linearly (FSBM work is linear in MBs, P:260)")
+        if me_only:
+            what = what.replace("ME+SME", "ME").split(" and ")[0] + (" (integer ME only)" if full else
+                                                                        ", extrapolated linearly")
         return {"value": fps, "unit": "frames/s", "cores": self.threads, "kind": "oracle",
                 "sample": f"{what}; {t:.1f} s wall on {self.threads} thread(s)",
                 "seconds": {"me": t1 - t0, "sme": t2 - t1, "int": t3 - t2, "total": t},
@@ -289,7 +295,8 @@ def run_reference(args, cfg):
 
 def config_json(cfg, args):
     return {"workload": cfg.name, "baseline_config_index": cfg.baseline_index, "width": cfg.width,
-            "height": cfg.height, "n_rf": cfg.n_rf, "sa_range": cfg.sa_range, "path": "int+me+sme (IPPP stream)",
+            "height": cfg.height, "n_rf": cfg.n_rf, "sa_range": cfg.sa_range,
+            "path": "integer FSBM ME only (me_estimate)" if cfg.path == "me" else "int+me+sme (IPPP stream)",
             "partitions": 41, "parallelism": f"mb-row x{args.gpus}" + (" adaptive" if args.adaptive else "") +
             (f" ({args.exchange} exchange)" if args.gpus > 1 and not args.adaptive else ""),
             "l2": "flushed (512 MiB write) before every timed step",
@@ -309,6 +316,91 @@ def _all_max(x):
         return h
     dist.all_reduce(x, op=dist.ReduceOp.MAX)
     return x
+
+
+def run_me_only(args, cfg, me, dev, feves):
+    """BASELINE configs 1-2 ("integer ME only" / "integer FSBM ME"): one step = me_estimate of frame
+    t over its n_rf previous frames (device resident, L2 flushed before each step); e2e = the same
+    through the C-ABI with the new frame uploaded from pinned host memory into a device ring and the
+    full-pel MVs + SADs downloaded, every step."""
+    import torch
+    from synth import ippp_sequence
+    n_frames = cfg.n_rf + 4
+    host = ippp_sequence(cfg.width, cfg.height, n_frames, 1000 + cfg.baseline_index)
+    frames = [torch.from_numpy(f).to(dev) for f in host]
+    pinned = [torch.from_numpy(f).pin_memory() for f in host]
+    flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
+    stream = torch.cuda.current_stream(dev)
+    out = me.new_mvs()
+
+    def step(t):
+        me.estimate(frames[t % n_frames], [frames[(t - 1 - k) % n_frames] for k in range(cfg.n_rf)], out=out)
+
+    for t in range(cfg.n_rf, cfg.n_rf + args.warmup):
+        step(t)
+    torch.cuda.synchronize()
+    me.set_timing(False)
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    clocks = Clocks(dev.index or 0)
+    clocks.start()
+    for k in range(args.steps):
+        flush.fill_(k & 0xff)
+        ev[k][0].record(stream)
+        step(cfg.n_rf + args.warmup + k)
+        ev[k][1].record(stream)
+    torch.cuda.synchronize()
+    ck = clocks.stop()
+    total_ms = sum(a.elapsed_time(b) for a, b in ev)
+    fps = args.steps / (total_ms / 1e3)
+    me.set_timing(True)
+    me_ms = []
+    for k in range(max(5, min(args.steps, 20))):
+        flush.fill_(k & 0xff)
+        step(cfg.n_rf + k)
+        me_ms.append(me.timings()[1])
+    launches = me.launches * args.steps
+    # e2e: device ring of n_rf + 1 frames, H2D of the new frame + D2H of the MVs / SADs inside the region
+    ring = [torch.empty_like(frames[0]) for _ in range(cfg.n_rf + 1)]
+    for i in range(cfg.n_rf):
+        ring[i].copy_(frames[i])
+    mv_h = torch.empty(me.mv_shape() + (2,), dtype=torch.int16).pin_memory()
+    sad_h = torch.empty(me.mv_shape(), dtype=torch.uint16).pin_memory()
+    torch.cuda.synchronize()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record(stream)
+    n_e2e = args.e2e_steps
+    for i in range(n_e2e):
+        t = cfg.n_rf + i
+        cur = ring[t % len(ring)]
+        cur.copy_(pinned[t % n_frames], non_blocking=True)
+        me.estimate(cur, [ring[(t - 1 - k) % len(ring)] for k in range(cfg.n_rf)], out=out)
+        mv_h.copy_(out[0], non_blocking=True)
+        sad_h.copy_(out[1], non_blocking=True)
+    e1.record(stream)
+    torch.cuda.synchronize()
+    e2e = {"value": n_e2e / (e0.elapsed_time(e1) / 1e3), "unit": "frames/s",
+           "h2d_bytes_per_step": pinned[0].numel(), "d2h_bytes_per_step": mv_h.numel() * 2 + sad_h.numel() * 2,
+           "api": "me_estimate (C-ABI) on a device frame ring, pinned host frame in, full-pel MVs + SADs out"}
+    u = workload_units(cfg)
+    pk, pk_src = peaks()
+    peak_px = N_SM * PX_PER_CLK_SM * pk.get("sm_max_mhz", 1965.0) * 1e6
+    me_mean = statistics.mean(me_ms)
+    achieved = u["me_px"] / (me_mean / 1e3)
+    return {
+        "metric": METRIC, "value": fps, "unit": "frames/s", "n_gpus": 1, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": total_ms / args.steps, "higher_is_better": True,
+        "scaling": "strong", "vs_baseline": None, "dtype": "u8",
+        "data": "synthetic (gen-tex: 8 sinusoids in (1.25,-0.75) px/frame motion + noise, seeded)",
+        "config": dict(config_json(cfg, args), graph="none"),
+        "candidate_gsad_per_s": u["me_cands"] * fps / 1e9, "px_absdiff_per_s": u["me_px"] * fps,
+        "kernels_ms": {"me": me_mean, "note": "CUDA events around the ME launch (library module timer)"},
+        "clocks": ck, "e2e": e2e, "gpu_launches": launches,
+        "roofline": {"bound": "alu", "kernel": f"me_fsbm_kernel<{cfg.sa_range}>", "work": "px-absdiffs of ME per launch",
+                     "achieved": achieved / 1e12, "peak": peak_px / 1e12, "unit": "Tpx-absdiff/s",
+                     "frac": achieved / peak_px, "traffic": None,
+                     "peak_source": f"148 SM x 64 VABSDIFF4 lanes/clk x 4 px x sm_max_mhz ({pk_src})"},
+        "cpu_baseline": None,
+    }
 
 
 def run_feves(args, cfg):
@@ -342,6 +434,12 @@ def run_feves(args, cfg):
             pm[:, r, 0], pm[:, r, 1] = round(-1.25 * (r + 1)), round(0.75 * (r + 1))
         pmv_dev = pm.to(dev)
         me.set_pmv(pmv_dev)
+    if cfg.path == "me" and world == 1 and not (args.lam or args.max_pmv):
+        line = run_me_only(args, cfg, me, dev, feves)
+        if not args.no_cpu_baseline:
+            line["cpu_baseline"] = cpu_baseline(cfg, args)
+        print(json.dumps(line), flush=True)
+        return
     r0, r1 = stripes(me.mb_rows, world)[rank]
     me.set_rows(r0, r1)      # (ShardedStream may re-split later in adaptive mode)
     for opt, val in ((me.OPT_PIPELINE_RF, args.pipeline), (me.OPT_ME_CTAS_PER_SM, args.me_ctas),

@@ -393,8 +393,18 @@ __global__ void __launch_bounds__(S_CT ? 128 : 256, S_CT ? FEVES_ME_MINB : 2) me
   const int dy_begin = -R + sub * DYL;
 
   // ---- CF MB -> shared memory (read back as broadcast LDS.128 rows) ----
-  for (int i = threadIdx.x; i < 64; i += blockDim.x)
-    cf_s[i] = load4_clamped(P.cf, P.W, P.H, 16 * mbx + 4 * (i & 3), 16 * mby + (i >> 2));
+  // Small SAs (S <= 32: one RF window of few candidates per CTA, latency-bound grids) keep the
+  // CF word in a register and store it after the first window's loads are issued, so the two
+  // global round trips overlap instead of serialising (the S = 64 / 128 kernels are unchanged).
+  constexpr bool kLateCf = S_CT > 0 && S_CT <= 32 && !FUSE;
+  uint32_t cf_w = 0;
+  if (kLateCf) {
+    if (threadIdx.x < 64)
+      cf_w = load4_clamped(P.cf, P.W, P.H, 16 * mbx + 4 * (threadIdx.x & 3), 16 * mby + (threadIdx.x >> 2));
+  } else {
+    for (int i = threadIdx.x; i < 64; i += blockDim.x)
+      cf_s[i] = load4_clamped(P.cf, P.W, P.H, 16 * mbx + 4 * (i & 3), 16 * mby + (i >> 2));
+  }
 
   const int xw0 = 16 * mbx - R, yw0 = 16 * mby - R;
   constexpr int NSTG = S_CT ? me_nstage(S_CT) : 1;      // window stagings per RF (dy halves)
@@ -476,6 +486,7 @@ __global__ void __launch_bounds__(S_CT ? 128 : 256, S_CT ? FEVES_ME_MINB : 2) me
                        __byte_perm(w[2], w[3], 0x6543), __byte_perm(w[3], w[4], 0x6543));
       }
     }
+    if (kLateCf && ref == 0 && threadIdx.x < 64) cf_s[threadIdx.x] = cf_w;
     __syncthreads();
 
     for (int c = hs * (DYL / NSTG); c < (hs + 1) * (DYL / NSTG); c += kMeT) {
