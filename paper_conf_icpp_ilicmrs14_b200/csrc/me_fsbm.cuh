@@ -397,10 +397,13 @@ __global__ void __launch_bounds__(S_CT ? 128 : 256, S_CT ? FEVES_ME_MINB : 2) me
   // CF word in a register and store it after the first window's loads are issued, so the two
   // global round trips overlap instead of serialising (the S = 64 / 128 kernels are unchanged).
   constexpr bool kLateCf = S_CT > 0 && S_CT <= 32 && !FUSE;
-  uint32_t cf_w = 0;
+  uint32_t cf_w[2] = {0, 0};                              // 64 words over 32 (S = 32) or 64 (S = 16) threads
   if (kLateCf) {
-    if (threadIdx.x < 64)
-      cf_w = load4_clamped(P.cf, P.W, P.H, 16 * mbx + 4 * (threadIdx.x & 3), 16 * mby + (threadIdx.x >> 2));
+#pragma unroll
+    for (int j = 0; j < 2; ++j) {
+      const int i = threadIdx.x + j * (int)blockDim.x;
+      if (i < 64) cf_w[j] = load4_clamped(P.cf, P.W, P.H, 16 * mbx + 4 * (i & 3), 16 * mby + (i >> 2));
+    }
   } else {
     for (int i = threadIdx.x; i < 64; i += blockDim.x)
       cf_s[i] = load4_clamped(P.cf, P.W, P.H, 16 * mbx + 4 * (i & 3), 16 * mby + (i >> 2));
@@ -486,7 +489,13 @@ __global__ void __launch_bounds__(S_CT ? 128 : 256, S_CT ? FEVES_ME_MINB : 2) me
                        __byte_perm(w[2], w[3], 0x6543), __byte_perm(w[3], w[4], 0x6543));
       }
     }
-    if (kLateCf && ref == 0 && threadIdx.x < 64) cf_s[threadIdx.x] = cf_w;
+    if (kLateCf && ref == 0) {
+#pragma unroll
+      for (int j = 0; j < 2; ++j) {
+        const int i = threadIdx.x + j * (int)blockDim.x;
+        if (i < 64) cf_s[i] = cf_w[j];
+      }
+    }
     __syncthreads();
 
     for (int c = hs * (DYL / NSTG); c < (hs + 1) * (DYL / NSTG); c += kMeT) {
