@@ -64,8 +64,8 @@ def parse():
     ap.add_argument("--overlap", type=int, default=None,
                     help="ME_OPT_OVERLAP_SME for the e2e stream (SME(t) co-runs with ME(t+1))")
     ap.add_argument("--exchange", choices=["peer", "collective"], default="peer",
-                    help="N>1: stripe+halo pull and SME stores over peer memory (PeerStream) or NCCL "
-                         "broadcast + gather (ShardedStream; always used with --adaptive)")
+                    help="N>1: stripe+halo pull and SME stores over peer memory ordered by stream flags "
+                         "(PeerStream) or NCCL broadcast + gather (ShardedStream)")
     return ap.parse_args()
 
 
@@ -298,7 +298,7 @@ def config_json(cfg, args):
             "height": cfg.height, "n_rf": cfg.n_rf, "sa_range": cfg.sa_range,
             "path": "integer FSBM ME only (me_estimate)" if cfg.path == "me" else "int+me+sme (IPPP stream)",
             "partitions": 41, "parallelism": f"mb-row x{args.gpus}" + (" adaptive" if args.adaptive else "") +
-            (f" ({args.exchange} exchange)" if args.gpus > 1 and not args.adaptive else ""),
+            (f" ({args.exchange} exchange)" if args.gpus > 1 else ""),
             "l2": "flushed (512 MiB write) before every timed step",
             "graph": "one CUDA graph per frame (ME_OPT_GRAPH)" if args.impl == "feves" and args.graph and args.gpus == 1
             else "none",
@@ -456,11 +456,11 @@ def run_feves(args, cfg):
     pinned = [torch.from_numpy(f).pin_memory() for f in host]
     buf = torch.empty_like(frames[0])
     flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
-    peer = world > 1 and args.exchange == "peer" and not args.adaptive
+    peer = world > 1 and args.exchange == "peer"
     if world == 1:
         ss = None
     elif peer:
-        ss = PeerStream(me)
+        ss = PeerStream(me, adaptive=args.adaptive)
     else:
         ss = ShardedStream(me, adaptive=args.adaptive)
 
@@ -517,7 +517,7 @@ def run_feves(args, cfg):
     per_rank = None
     if peer:                                         # each rank's device time per push (CUDA events)
         ms = ss.stripe_ms()[-args.steps:]
-        mine = {"rank": rank, "rows": list(stripes(me.mb_rows, world)[rank]), "stripe_ms_mean": statistics.mean(ms)}
+        mine = {"rank": rank, "rows": list(ss.cur[rank]), "stripe_ms_mean": statistics.mean(ms)}
         per_rank = [None] * world
         dist.all_gather_object(per_rank, mine)
     mod_ms, mod, _ = timed(max(5, min(args.steps, 20)), True)

@@ -75,8 +75,9 @@ class AdaptiveSplit:
     def stripes(self):
         return list(self.cur)
 
-    def update(self, times):
-        rows = [r1 - r0 for r0, r1 in self.cur]
+    def update(self, times, split=None):
+        """times[i] = device i's time for a frame computed with ``split`` (default: the current one)"""
+        rows = [r1 - r0 for r0, r1 in (self.cur if split is None else split)]
         k_now = [max(t, 1e-9) / max(m, 1) for t, m in zip(times, rows)]
         self.K = k_now if self.K is None else [self.alpha * a + (1 - self.alpha) * b
                                                for a, b in zip(self.K, k_now)]
@@ -205,19 +206,31 @@ class PeerStream:
     ready flag is written only after rank src passed the done-waits of frame t and whatever its
     caller enqueued after push t (e.g. the D2H of frame t's outputs).  The tensors returned on
     rank src are complete in its stream order and stay valid until push t+2.  Results equal
-    the single-GPU stream bitwise (pin P11); the split is the static equidistant one.
-    ``stripe_ms()`` gives each push's device time on this rank (CUDA events)."""
+    the single-GPU stream bitwise (pin P11).  ``stripe_ms()`` gives each push's device time on
+    this rank (CUDA events).
 
-    def __init__(self, me, group=None, src: int = 0):
+    Split: equidistant, or with ``adaptive=True`` the paper's iterative phase (Alg. 1
+    l.7-11) through ``AdaptiveSplit``: at push t every rank reads its own
+    device time of frame t - ``lag`` (an event pair two frames old, so no stall on the frame in
+    flight), the times are all-gathered over a CPU (gloo) group, and every rank applies the same
+    new split to frame t.  Ranks then pull whole frames (no halo-only copies: a grown stripe needs
+    rows a halo-only ring frame would lack); the library refreshes the SF rows a moved stripe
+    reads.  ``timer(rank, rows, seconds) -> seconds`` may replace the measured time (tests)."""
+
+    def __init__(self, me, group=None, src: int = 0, adaptive: bool = False, lag: int = 2, timer=None):
         import paper_conf_icpp_ilicmrs14_b200 as F
         self.F = F
         self.me, self.group, self.src = me, group, src
         self.rank = dist.get_rank(group)
         self.world = dist.get_world_size(group)
+        self.split = AdaptiveSplit(me.mb_rows, self.world) if adaptive else None
+        self.lag, self.timer = lag, timer
+        self.ctrl = dist.new_group(backend="gloo") if adaptive else None   # CPU control plane (P:50)
         self.cur = stripes(me.mb_rows, self.world)
+        self.history = []                                                    # split used per frame
         r0, r1 = self.cur[self.rank]
         me.set_rows(r0, r1)
-        me.set_option(me.OPT_HALO_ONLY, 1)
+        me.set_option(me.OPT_HALO_ONLY, 0 if adaptive else 1)
         dev = me.device
         H, W = me.height, me.width
         shape = (me.mb_rows, me.mb_cols, me.n_rf, 41)
@@ -267,6 +280,19 @@ class PeerStream:
                 self.frames[b].copy_(frame.view(self.me.height, self.me.width), non_blocking=True)
                 for p in self.ready_ptrs:
                     F.stream_write_value(self.pub, p + 4 * b, t + 1)
+        if self.split is not None and t >= self.lag:                         # Alg. 1 iterative phase
+            k = t - self.lag
+            a, z = self.times[k]
+            z.synchronize()                                                  # frame t - lag: normally done
+            secs = a.elapsed_time(z) / 1e3
+            r0k, r1k = self.history[k][self.rank]
+            if self.timer is not None:
+                secs = self.timer(self.rank, r1k - r0k, secs)
+            allt = [torch.zeros(1, dtype=torch.float64) for _ in range(self.world)]
+            dist.all_gather(allt, torch.tensor([secs], dtype=torch.float64), group=self.ctrl)
+            self.cur = self.split.update([float(x) for x in allt], split=self.history[k])
+            self.me.set_rows(*self.cur[self.rank])
+        self.history.append(list(self.cur))
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record(cs)
         r0 = self.cur[self.rank][0]

@@ -91,7 +91,11 @@ def test_two_rank_sharded_stream_equals_oracle(adaptive):
         assert history[0] == [(0, 4), (4, 8)] and history[-1] == [(0, 6), (6, 8)]
 
 
-def _peer_worker(rank, world, port, q, host_frames):
+def _slow_rank1_time(rank, rows, secs):
+    return (3.0 if rank == 1 else 1.0) * rows
+
+
+def _peer_worker(rank, world, port, q, host_frames, adaptive=False):
     import torch.distributed as dist
     os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
     dist.init_process_group("gloo", rank=rank, world_size=world)
@@ -101,7 +105,7 @@ def _peer_worker(rank, world, port, q, host_frames):
         from synth import gen_tex
         torch.cuda.set_device(0)
         me = F.MotionEstimator(W, H, S, N_RF)
-        ps = PeerStream(me)
+        ps = PeerStream(me, adaptive=adaptive, timer=_slow_rank1_time if adaptive else None)
         frames_np = [gen_tex(W, H, t, 37) for t in range(N_FRAMES)]
         frames = [torch.from_numpy(f) for f in frames_np]
         frames = [f.pin_memory() if host_frames else f.cuda() for f in frames]
@@ -114,7 +118,7 @@ def _peer_worker(rank, world, port, q, host_frames):
         ps.close()
         if rank == 0:
             ok = _oracle_matches(outs, frames_np)
-            q.put(ok)
+            q.put((ok, ps.history) if adaptive else ok)
     finally:
         dist.destroy_process_group()
 
@@ -157,3 +161,24 @@ def test_halo_only_push_refuses_missing_rows():
     me.set_rows(0, 2)                   # the original stripe still works
     me.stream_push(frames[2])
     torch.cuda.synchronize()
+
+
+def test_adaptive_peer_stream_equals_oracle():
+    """f3 on the flag-ordered peer exchange: rank 1 reports 3x the time per MB row, so from frame
+    lag = 2 on the split moves rows to rank 0 (Alg. 1's iterative phase, P:50; K_i per row, P:218);
+    every frame's assembled output still equals the oracle (pin P11 + the library's SF refresh)."""
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    with socket.socket() as s:
+        s.bind(("127.0.0.1", 0))
+        port = s.getsockname()[1]
+    procs = [ctx.Process(target=_peer_worker, args=(r, 2, port, q, False, True)) for r in range(2)]
+    for p in procs:
+        p.start()
+    ok, history = q.get(timeout=600)
+    for p in procs:
+        p.join(timeout=120)
+        assert p.exitcode == 0
+    assert ok
+    assert history[0] == [(0, 4), (4, 8)] and history[1] == [(0, 4), (4, 8)]
+    assert history[-1] == [(0, 6), (6, 8)]

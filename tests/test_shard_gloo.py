@@ -233,3 +233,17 @@ def test_adaptive_sharded_stream_moves_rows_and_stays_exact(orc):
         oq, os_ = orc.sme(frames[t], rfs, mv)
         np.testing.assert_array_equal(qm.reshape(n, N_RF, 41, 2)[:, :n_ref], oq)
         np.testing.assert_array_equal(qs.reshape(n, N_RF, 41)[:, :n_ref], os_)
+
+
+def test_adaptive_split_with_a_lagged_split():
+    """AdaptiveSplit.update(times, split=...) charges the times to the split that produced them
+    (PeerStream adapts with a lag of two frames, by when the split may already have moved):
+    K_i = t_i / m_i per row, next m_i proportional to 1 / K_i (eq. (1))."""
+    from paper_conf_icpp_ilicmrs14_b200.shard import AdaptiveSplit
+    a = AdaptiveSplit(8, 2, smoothing=0.0)
+    assert a.stripes() == [(0, 4), (4, 8)]
+    old = a.stripes()
+    a.update([4.0, 4.0], split=[(0, 2), (2, 8)])        # 2 rows in 4 s vs 6 rows in 4 s: K = 2, 2/3
+    assert a.stripes() == [(0, 2), (2, 8)]
+    a.update([1.0, 3.0], split=old)                     # K = 1/4, 3/4 -> 3:1
+    assert a.stripes() == [(0, 6), (6, 8)]
