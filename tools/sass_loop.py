@@ -30,15 +30,18 @@ def main():
         m = re.match(r"\s+/\*([0-9a-f]{4,5})\*/\s+(@!?U?P\w+\s+)?([A-Z0-9_.]+)([^;]*);", l)
         if m:
             ins.append((int(m.group(1), 16), m.group(3), m.group(4)))
-    best = None
+    loops = []
     for a, op, args in ins:
         if op.startswith("BRA"):
             t = re.search(r"0x([0-9a-f]+)", args)
             if t and int(t.group(1), 16) < a:
-                span = a - int(t.group(1), 16)
-                if best is None or span > best[1] - best[0]:
-                    best = (int(t.group(1), 16), a)
-    lo, hi = best
+                loops.append((int(t.group(1), 16), a))
+    # the hottest loop = the innermost loop holding the most ALU work per instruction
+    def density(lh):
+        body = [op for a, op, _ in ins if lh[0] <= a <= lh[1]]
+        n_alu = sum(1 for op in body if op.split(".")[0] in ALU and not op.startswith("IMAD"))
+        return n_alu / max(1, len(body)), -len(body)
+    lo, hi = max(loops, key=density)
     loop = [(a, op) for a, op, _ in ins if lo <= a <= hi]
     c = collections.Counter(op for _, op in loop)
     alu = sum(v for k, v in c.items() if k.split(".")[0] in ALU and not k.startswith("IMAD"))
