@@ -460,7 +460,21 @@ def run_feves(args, cfg):
     if world == 1:
         ss = None
     elif peer:
-        ss = PeerStream(me, adaptive=args.adaptive)
+        # the flag-ordered peer exchange needs CUDA IPC + stream memory operations between the
+        # ranks' GPUs; if the platform refuses either (checked collectively at setup), fall back to
+        # the NCCL broadcast / gather exchange and say so in the line
+        try:
+            ss = PeerStream(me, adaptive=args.adaptive)
+            ok = 1
+        except Exception as e:                       # noqa: BLE001 -- any setup failure -> fallback
+            print(f"PeerStream unavailable on this platform ({e}); using ShardedStream", file=sys.stderr)
+            ok = 0
+        flag = torch.tensor([ok], dtype=torch.int32, device=dev)
+        dist.all_reduce(flag, op=dist.ReduceOp.MIN)
+        if not int(flag.item()):
+            peer = False
+            args.exchange = "collective (peer exchange unavailable)"
+            ss = ShardedStream(me, adaptive=args.adaptive)
     else:
         ss = ShardedStream(me, adaptive=args.adaptive)
 

@@ -247,6 +247,28 @@ class PeerStream:
         allx = [None] * self.world
         dist.all_gather_object(allx, mine, group=group)
         self.opened = []
+        self.t = 0
+        self.times = []
+        err = None
+        try:                                          # mapping + a stream-memory-operation probe
+            self._map(allx, bufs if self.rank == src else None, dev)
+        except Exception as e:                        # noqa: BLE001 -- reported collectively below
+            err = e
+        ok = torch.tensor([0 if err else 1], dtype=torch.int32,
+                          device=dev if dist.get_backend(group) == "nccl" else "cpu")
+        dist.all_reduce(ok, op=dist.ReduceOp.MIN, group=group)
+        if not int(ok.item()):                        # every rank raises: the caller can fall back
+            for p in self.opened:
+                try:
+                    me.ipc_close(p)
+                except Exception:                     # noqa: BLE001
+                    pass
+            self.opened = []
+            raise F.FevesError(f"PeerStream unavailable: {err or 'a peer rank failed'}")
+        dist.barrier(group=group)
+
+    def _map(self, allx, bufs, dev):
+        me, src = self.me, self.src
 
         def open_(h):
             p = me.ipc_open(*h)
@@ -262,9 +284,12 @@ class PeerStream:
             ptrs = [open_(h) for h in allx[src][1:]]
         self.f_ptr, self.qm_ptr, self.qs_ptr = ptrs[0:2], ptrs[2:4], ptrs[4:6]
         self.done_ptr = ptrs[6]                                              # rank src's done words
-        self.t = 0
-        self.times = []
-        dist.barrier(group=group)
+        # probe: a stream write into rank src's memory and a stream wait on local memory (raises
+        # if this platform does not support stream memory operations on peer-mapped memory)
+        probe = torch.cuda.current_stream(dev)
+        self.F.stream_write_value(probe, self.done_ptr + 4 * self.rank, 0)
+        self.F.stream_wait_value(probe, self.ready.data_ptr(), 0)
+        probe.synchronize()
 
     def push(self, frame, frame_buf=None):
         """frame: this step's frame on rank ``src`` (device or pinned host tensor [H, W]);
