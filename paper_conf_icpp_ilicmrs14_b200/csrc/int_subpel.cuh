@@ -211,8 +211,15 @@ __global__ void __launch_bounds__(128, FEVES_INT_MINB) int_subpel_kernel(const I
 // coalesced 4-byte loads (each source word is read by 6 rows x 1.5 groups in the per-thread
 // kernel), then every thread reads its 6 x 6 words with LDS.128 + LDS.64 (its window starts
 // 16-byte aligned in the tile, so a warp's quarter-requests are bank-conflict free).
-constexpr int kIntTx = 8, kIntTy = 16;
-constexpr int kIntSrcRows = kIntTy + 5, kIntSrcWords = 4 * kIntTx + 2, kIntStride = 36;   // words per tile row
+#ifndef FEVES_INT_TX
+#define FEVES_INT_TX 8
+#endif
+#ifndef FEVES_INT_TY
+#define FEVES_INT_TY 16
+#endif
+constexpr int kIntTx = FEVES_INT_TX, kIntTy = FEVES_INT_TY;
+constexpr int kIntSrcRows = kIntTy + 5, kIntSrcWords = 4 * kIntTx + 2;
+constexpr int kIntStride = (kIntSrcWords + 3) & ~3;                                          // words per tile row
 static_assert(kIntStride >= kIntSrcWords && kIntStride % 4 == 0, "INT tile row stride");
 
 #ifndef FEVES_INT_TPC
