@@ -71,7 +71,10 @@ __host__ __device__ constexpr int me_nsub(int S) { return 32 / me_lx(S); }
 // warps splitting the dy range: at S = 16 (CIF, 396 MBs, one RF) a second warp takes the
 // other half of the dy range, doubling the warps of a grid too small to fill the GPU
 // (ME 10.9 -> 9.0 us).  Measured slower for S = 32 (69.9 -> 73.4 us), so only S = 16.
-__host__ __device__ constexpr int me_nwy(int S) { return S == 16 ? 2 : 1; }
+#ifndef FEVES_ME_NWY64
+#define FEVES_ME_NWY64 1
+#endif
+__host__ __device__ constexpr int me_nwy(int S) { return S == 16 ? 2 : S == 64 ? FEVES_ME_NWY64 : 1; }
 __host__ __device__ constexpr int me_dyl(int S) {
   return ((S + me_nsub(S) * me_nwy(S) - 1) / (me_nsub(S) * me_nwy(S)) + kMeT - 1) / kMeT * kMeT;
 }
