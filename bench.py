@@ -49,8 +49,10 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-budget", type=float, default=10.0,
                     help="reference arm: seconds of oracle wall time per step (a seeded MB sample)")
-    ap.add_argument("--cpu-frame", choices=["full", "sample"], default="full",
-                    help="cpu_baseline: the oracle on ONE FULL frame on all host cores (default) or a sample")
+    ap.add_argument("--cpu-frame", choices=["auto", "full", "sample"], default="auto",
+                    help="cpu_baseline: the oracle on ONE FULL frame on all host cores, or a seeded MB sample "
+                         "(auto: full when the calibrated estimate is <= --cpu-full-max seconds)")
+    ap.add_argument("--cpu-full-max", type=float, default=90.0)
     ap.add_argument("--sme-kernel", type=int, default=None, help="ME_OPT_SME_KERNEL (0 global-load, 1 staged)")
     ap.add_argument("--graph", type=int, default=1,
                     help="ME_OPT_GRAPH: one CUDA graph per frame (default 1; 0 = multi-stream enqueue)")
@@ -253,10 +255,14 @@ def cpu_baseline(cfg, args):
     """cpu_baseline of the bench line: the oracle on one full frame on all host cores
     (measured, not extrapolated), plus a single-thread timing on one MB row of it."""
     s = OracleSampler(cfg)
-    cb = s.run(s.n_total if args.cpu_frame == "full" else s.size_for(args.cpu_budget))
+    full = args.cpu_frame == "full"
+    if args.cpu_frame == "auto":
+        s.calibrate()                           # one MB per thread
+        full = s.t_cal * s.n_total / s.threads <= args.cpu_full_max
+    cb = s.run(s.n_total if full else s.size_for(args.cpu_budget))
     one = OracleSampler(cfg, threads=1)
     mbc = -(-cfg.width // 16)
-    st = one.run(mbc)                       # a seeded sample of one MB row's worth of MBs
+    st = one.run(min(mbc, one.size_for(10.0)))   # a seeded sample: one MB row's worth, at most ~10 s
     cb["single_thread"] = {"value": st["value"], "unit": "frames/s", "cores": 1, "sample": st["sample"],
                            "speedup_all_cores": cb["value"] / st["value"]}
     return cb
@@ -694,7 +700,8 @@ def run_feves(args, cfg):
         cpu = cpu_baseline(cfg, args)
     line = {
         "metric": METRIC, "value": fps, "unit": "frames/s", "n_gpus": world, "steps": args.steps,
-        "warmup": args.warmup, "ms_per_step": total_ms / args.steps, "higher_is_better": True,
+        "warmup": args.warmup, "ms_per_step": total_ms / args.steps,
+        "ms_per_step_median": statistics.median(step_ms), "higher_is_better": True,
         "scaling": "strong", "vs_baseline": None, "dtype": "u8",
         "data": "synthetic (gen-tex: 8 sinusoids in (1.25,-0.75) px/frame motion + noise, seeded)",
         "config": config_json(cfg, args),
