@@ -112,6 +112,39 @@ __device__ __forceinline__ int mode_part_rt(int m, int bx, int by) {
   }
 }
 
+// The 8 ring candidates' partition costs t_k (spiral order k, G14) in ONE pass: key = t_k * 8 + k,
+// min over the 8 keys (3-input mins), and an update of (best, bvx, bvy) iff min t < best -- the
+// same result as the ordered strict-< scan (the first of equal minima wins).  The 8 strip sums
+// are xor-shuffled as 4 packed 16-bit pairs (a strip partial SAD <= 16 rows x 4 px x 255 = 16320,
+// a partition sum <= 65280: no carry between the halves).  step = 2 (half stage) or 1 (quarter).
+template <bool RD>
+__device__ __forceinline__ void ring_update(const uint32_t (&v)[8], int xm, int step, int ox, int oy, int lambda,
+                                            int qpx, int qpy, uint32_t& best, int& bvx, int& bvy) {
+  uint32_t key[8];
+#pragma unroll
+  for (int i = 0; i < 4; ++i) {
+    uint32_t pk = v[2 * i] | (v[2 * i + 1] << 16);
+    const uint32_t a = __shfl_xor_sync(0xffffffffu, pk, 1);
+    pk += a & (0u - (uint32_t)(xm & 1));
+    const uint32_t b = __shfl_xor_sync(0xffffffffu, pk, 2);
+    pk += b & (0u - (uint32_t)((xm >> 1) & 1));
+#pragma unroll
+    for (int h = 0; h < 2; ++h) {
+      const int k = 2 * i + h;
+      uint32_t t = h ? (pk >> 16) : (pk & 0xffffu);
+      if (RD) t += lambda * (se_bits(ox + step * c_ring1[k][0] - qpx) + se_bits(oy + step * c_ring1[k][1] - qpy));
+      key[k] = t * 8u + (uint32_t)k;
+    }
+  }
+  const uint32_t m = min(min(min(key[0], key[1]), min(key[2], key[3])), min(min(key[4], key[5]), min(key[6], key[7])));
+  if ((m >> 3) < best) {
+    const int k = (int)(m & 7u);
+    best = m >> 3;
+    bvx = ox + step * ((int)((0x8885u >> (2 * k)) & 3u) - 1);   // ring-1 dx + 1 = 1,1,0,2,0,2,0,2
+    bvy = oy + step * ((int)((0xA508u >> (2 * k)) & 3u) - 1);   // ring-1 dy + 1 = 0,2,0,0,1,1,2,2
+  }
+}
+
 // partition sum over the strip lanes it spans (xm = its bx bits, warp-uniform); branch-free
 // (both shuffles always, masked adds), the compiler cannot see that xm is warp-uniform
 __device__ __forceinline__ uint32_t xsum_u(uint32_t v, int xm) {
@@ -204,14 +237,7 @@ __device__ __forceinline__ void refine_mode_s(const SmeParams& P, const Box& B, 
           jw = jn;
         }
       }
-      const int ox = bvx, oy = bvy;
-#pragma unroll
-      for (int k = 0; k < 8; ++k) {                 // spiral order, strict < (G14)
-        const int vx = ox + 2 * c_ring1[k][0], vy = oy + 2 * c_ring1[k][1];
-        uint32_t t = xsum_u(sad[k], xm);
-        if (RD) t += P.lambda * (se_bits(vx - qpx) + se_bits(vy - qpy));
-        if (t < best) { best = t; bvx = vx; bvy = vy; }
-      }
+      ring_update<RD>(sad, xm, 2, bvx, bvy, P.lambda, qpx, qpy, best, bvx, bvy);
     }
     // ---- quarter stage around the best half position (half-grid coordinates) ----
     {
@@ -243,14 +269,7 @@ __device__ __forceinline__ void refine_mode_s(const SmeParams& P, const Box& B, 
           oc = ocn;
         }
       }
-      const int ox = bvx, oy = bvy;
-#pragma unroll
-      for (int k = 0; k < 8; ++k) {                 // spiral order, strict < (G14)
-        const int vx = ox + c_ring1[k][0], vy = oy + c_ring1[k][1];
-        uint32_t t = xsum_u(qs[k], xm);
-        if (RD) t += P.lambda * (se_bits(vx - qpx) + se_bits(vy - qpy));
-        if (t < best) { best = t; bvx = vx; bvy = vy; }
-      }
+      ring_update<RD>(qs, xm, 1, bvx, bvy, P.lambda, qpx, qpy, best, bvx, bvy);
     }
     if (writer && (bx & xm) == 0) {
       P.out_qmvs[o + p] = (uint32_t)(uint16_t)bvx | ((uint32_t)(uint16_t)bvy << 16);
