@@ -453,7 +453,7 @@ def run_feves(args, cfg):
                      (me.OPT_SME_KERNEL, args.sme_kernel)):
         if val is not None:
             me.set_option(opt, val)
-    me.set_timing(True)
+    me.set_timing(False)                 # as in the timed pass: the graphs captured during the fill are its own
     stream = torch.cuda.current_stream(dev)
 
     n_frames = cfg.n_rf + 4
@@ -609,6 +609,18 @@ def run_feves(args, cfg):
         me.estimate(frames[t % n_frames], rf_list, out=mvs_scratch)
         me_only.append(me.timings()[1])
     del mvs_scratch
+    # f2 mode decision on the stream's last quarter-pel outputs (device resident)
+    md_ms = None
+    if world == 1:
+        md = []
+        for k in range(10):
+            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a.record(stream)
+            me.mode_decision(out_dev[0], out_dev[1])
+            b.record(stream)
+            md.append((a, b))
+        torch.cuda.synchronize()
+        md_ms = statistics.median(a.elapsed_time(b) for a, b in md)
 
     u = workload_units(cfg)
     int_ms = statistics.mean(m[0] for m in mod)
@@ -702,6 +714,7 @@ def run_feves(args, cfg):
         "metric": METRIC, "value": fps, "unit": "frames/s", "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": total_ms / args.steps,
         "ms_per_step_median": statistics.median(step_ms), "higher_is_better": True,
+        "step_ms": [round(x, 4) for x in step_ms] if os.environ.get("FEVES_BENCH_STEPS") else None,
         "scaling": "strong", "vs_baseline": None, "dtype": "u8",
         "data": "synthetic (gen-tex: 8 sinusoids in (1.25,-0.75) px/frame motion + noise, seeded)",
         "config": config_json(cfg, args),
@@ -709,7 +722,7 @@ def run_feves(args, cfg):
         "px_absdiff_per_s": (u["me_px"] + u["sme_px"]) * fps,
         "kernels_ms": {"int": int_ms, ("me_sme_fused" if fused else "me"): me_ms, "sme": sme_ms,
                        "int_isolated": int_iso_ms, "int_isolated_clean_l2": int_iso_clean_ms,
-                       "int_stateless_all_rf": int_stateless_ms,
+                       "int_stateless_all_rf": int_stateless_ms, "mode_decision": md_ms,
                        "me_only_isolated": me_only_ms,
                        "note": "CUDA events around each launch on its own stream" + (
                            "; fused: INT(t-1) then one ME+SME kernel" if fused else

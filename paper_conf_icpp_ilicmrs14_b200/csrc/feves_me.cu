@@ -1049,8 +1049,8 @@ extern "C" int me_set_timing(me_ctx* c, int on) {
   if (on && !c->ev_t[0])
     for (int i = 0; i < 6; ++i)
       if (cudaEventCreate(&c->ev_t[i]) != cudaSuccess) { cudaGetLastError(); return ME_ENOMEM; }
+  if (c->timing != (on ? 1 : 0)) c->gepoch++;           // captured stream graphs hold the timer nodes
   c->timing = on ? 1 : 0;
-  c->gepoch++;
   return ME_OK;
 }
 
