@@ -194,32 +194,6 @@ struct SumKeys { static constexpr bool value = S_CT > 0 && S_CT <= 128 && KSH ==
 template <int S_CT, int KSH>
 struct QuadKeys { static constexpr bool value = SumKeys<S_CT, KSH>::value && S_CT == 128; };
 
-#ifndef FEVES_ME_INV_ARITH
-#define FEVES_ME_INV_ARITH 0
-#endif
-// Inverse of the DENSE spiral rank over the SA [-R, R-1]^2 (G1, G4): rings l <= R-1 are complete
-// (dense rank = spiral rank: ring l starts at (2l-1)^2, first the pairs (x,-l),(x,+l) for
-// x = -l+1..l-1, then (-l,y),(+l,y) for y = -l..l); of ring R only x = -R or y = -R lie in the SA:
-// (x,-R) for x = -R+1..R-1, then (-R,y) for y = -R..R-1.  Returns (dx & 0xffff) | (dy << 16).
-__device__ __forceinline__ uint32_t dense_rank_to_mv(uint32_t r, int R) {
-  int dx, dy;
-  const int full = (2 * R - 1) * (2 * R - 1);
-  if ((int)r < full) {
-    int l = ((int)sqrtf((float)r) + 1) >> 1;                // (2l-1)^2 <= r < (2l+1)^2
-    if ((2 * l + 1) * (2 * l + 1) <= (int)r) ++l;
-    if (l > 0 && (2 * l - 1) * (2 * l - 1) > (int)r) --l;
-    const int off = (int)r - (2 * l - 1) * (2 * l - 1);
-    if (l == 0) { dx = 0; dy = 0; }
-    else if (off < 2 * (2 * l - 1)) { dx = -l + 1 + (off >> 1); dy = (off & 1) ? l : -l; }
-    else { const int o2 = off - 2 * (2 * l - 1); dy = -l + (o2 >> 1); dx = (o2 & 1) ? l : -l; }
-  } else {
-    const int o = (int)r - full;
-    if (o < 2 * R - 1) { dx = -R + 1 + o; dy = -R; }
-    else { dx = -R; dy = -R + (o - (2 * R - 1)); }
-  }
-  return (uint32_t)(uint16_t)dx | ((uint32_t)(uint16_t)dy << 16);
-}
-
 __host__ __device__ constexpr int part_log2n(int p) {   // log2(number of 4x4 blocks of partition p, G7)
   return p == 0 ? 4 : p < 5 ? 3 : p < 9 ? 2 : p < 25 ? 1 : 0;
 }
@@ -624,11 +598,7 @@ __global__ void __launch_bounds__(S_CT ? 128 : 256, S_CT ? FEVES_ME_MINB : 2) me
         rk = SumKeys<S_CT, KSH>::value ? (k & 0xffffu) >> part_log2n(p) : k & ((1u << KSH) - 1u);
         sad = k >> KSH;                                      // J = SAD + lambda*R(mv) (G18)
       }
-      uint32_t mv;                                           // SA offset (dx, dy)
-      if (FEVES_ME_INV_ARITH && S_CT > 0 && !QUAD && KSH == 16 && !kPmv)
-        mv = dense_rank_to_mv(rk, S_CT / 2);                 // arithmetic inverse: no global round trip
-      else
-        mv = __ldg(P.inv_tab + rk);
+      uint32_t mv = __ldg(P.inv_tab + rk);                   // SA offset (dx, dy)
       if (KSH != 16)                                         // rate of the offset = R(mv - p) (G21)
         sad -= (uint32_t)(P.lambda * (se_bits(4 * (int)(int16_t)(mv & 0xffffu)) + se_bits(4 * (int)(int16_t)(mv >> 16))));
       if (kPmv && P.pmv)                                     // mv = p + offset (G21)
