@@ -145,15 +145,6 @@ __device__ __forceinline__ void ring_update(const uint32_t (&v)[8], int xm, int 
   }
 }
 
-// partition sum over the strip lanes it spans (xm = its bx bits, warp-uniform); branch-free
-// (both shuffles always, masked adds), the compiler cannot see that xm is warp-uniform
-__device__ __forceinline__ uint32_t xsum_u(uint32_t v, int xm) {
-  const uint32_t a = __shfl_xor_sync(0xffffffffu, v, 1);
-  v += a & (0u - (uint32_t)(xm & 1));
-  const uint32_t b = __shfl_xor_sync(0xffffffffu, v, 2);
-  return v + (b & (0u - (uint32_t)((xm >> 1) & 1)));
-}
-
 // TMA bulk copy global -> shared (16-byte aligned, size a multiple of 16), completing on an
 // mbarrier (transaction bytes), and the mbarrier helpers
 __device__ __forceinline__ void bulk_g2s(uint32_t dst, const void* src, uint32_t bytes, uint32_t bar) {
