@@ -33,25 +33,29 @@ struct IntParams {
 // Two columns per 32-bit register, one per 16-bit lane, and every lane kept
 // NON-NEGATIVE so plain 32-bit IADD/IMAD are exact per lane (no carry or
 // borrow can cross lanes).  A 6-tap result x1 in [-2550, 10710] is carried as
-// x1 + 2560 in [10, 13270]; 2560 = 80 * 32 cancels exactly in the >>5 and
-// >>10 roundings.  (No 16x2 subtraction: ptxas was seen to
+// x1 + B in [5658, 18918], B = 8208 = 256 * 32 + 16: the +16 is the rounding of
+// (x1 + 16) >> 5, and 32 * B = 256 * 1024 + 512 is exactly the rounding of
+// (j1 + 512) >> 10 plus 256 (j1 = the tap sum of six biased h1), so both
+// shifted values come out as (rounded value) + 256 and the Clip1 to [0, 255] is
+// a clamp to [256, 511] whose LOW BYTE is the sample -- no rounding add and no
+// bias subtraction.  (No 16x2 subtraction: ptxas was seen to
 // miscompile __vsub2 when one lane is dead.)
-constexpr uint32_t kBias = 2560u;
+constexpr uint32_t kBias = 8208u;
 constexpr uint32_t kBias2 = kBias | (kBias << 16);
-// tap6 on packed byte columns: (a+f) - 5(b+e) + 20(c+d) + 2560, per lane
+// tap6 on packed byte columns: (a+f) - 5(b+e) + 20(c+d) + B, per lane
 __device__ __forceinline__ uint32_t tap6x2b(uint32_t a, uint32_t b, uint32_t c, uint32_t d, uint32_t e, uint32_t f) {
   const uint32_t s = a + f, q = b + e, m = c + d;                   // lanes <= 510: no carry
-  return (m * 20u + s) + (kBias2 - q * 5u);                          // lanes in [10, 13270]
+  return (m * 20u + s) + (kBias2 - q * 5u);                          // lanes in [5658, 18918]
 }
-// Clip1((x1 + 16) >> 5) on two biased lanes -> two u16 lanes in [0, 255]
+// Clip1((x1 + 16) >> 5) + 256 on two biased lanes: u16 lanes in [256, 511], low byte = sample
 __device__ __forceinline__ uint32_t clip_half2(uint32_t vb) {
-  const uint32_t t = ((vb + 0x00100010u) >> 5) & 0x07ff07ffu;       // ((x1+16)>>5) + 80 per lane
-  return __vminu2(__vmaxu2(t, 0x00500050u), 0x014f014fu) - 0x00500050u;   // clamp to [80, 335], -80
+  const uint32_t t = (vb >> 5) & 0x07ff07ffu;                       // ((x1+16)>>5) + 256 per lane
+  return __vminu2(__vmaxu2(t, 0x01000100u), 0x01ff01ffu);
 }
 __device__ __forceinline__ int lo_u16(uint32_t x) { return (int)(x & 0xffffu); }
 __device__ __forceinline__ int hi_u16(uint32_t x) { return (int)(x >> 16); }
-// j = Clip1((j1 + 512) >> 10) from the biased sum jb = j1 + 32 * 2560
-__device__ __forceinline__ uint32_t clip_j(int jb) { return (uint32_t)min(max(jb - (32 * (int)kBias - 512), 0) >> 10, 255); }
+// Clip1((j1 + 512) >> 10) + 256 from the biased sum jb = j1 + 32 * B (> 0): low byte = j
+__device__ __forceinline__ uint32_t clip_j(int jb) { return (uint32_t)min(max(jb >> 10, 256), 511); }
 
 // low bytes of four u16 lanes (pairs a, b) -> one byte word
 __device__ __forceinline__ uint32_t bytes_of(uint32_t a, uint32_t b) { return __byte_perm(a, b, 0x6420); }
@@ -97,7 +101,7 @@ __device__ __forceinline__ void int_compute(const IntParams& P, int g, int rr, c
   // j1 = tap6 over h1 at columns c-2..c+3 (int32), c = 4..19
   int hv[22];
 #pragma unroll
-  for (int j = 1; j < 12; ++j) { hv[2 * j - 2] = lo_u16(h1[j]); hv[2 * j - 1] = hi_u16(h1[j]); }   // hv[i] = h1 + 2560 at c = i+2
+  for (int j = 1; j < 12; ++j) { hv[2 * j - 2] = lo_u16(h1[j]); hv[2 * j - 1] = hi_u16(h1[j]); }   // hv[i] = h1 + B at c = i+2
   uint32_t jb[16];
 #pragma unroll
   for (int i = 0; i < 16; ++i) {   // output column c = i+4: h1 at c-2..c+3 = hv[i .. i+5]
@@ -236,17 +240,38 @@ __global__ void __launch_bounds__(kIntTx * kIntTy) int_tile_kernel(const IntPara
   const int xs = 16 * g0 - P.pad - 4;                      // frame column of tile word 0
   const int tid = threadIdx.y * kIntTx + threadIdx.x;
   const bool fast = P.vec_ok && xs >= 0 && xs + 4 * kIntSrcWords <= P.W;
-  // stage the source tile of tile row ty (plane rows r0 .. r0+15) into buffer b
+  // stage the source tile of tile row ty (plane rows r0 .. r0+15) into buffer b.  Border tiles
+  // with aligned rows (vec_ok: W % 4 == 0, so a word is wholly inside or wholly outside the
+  // frame) copy the frame's edge word in place of every outside word, and edge_fix() then
+  // replicates its edge byte (G5 clamp) -- all loads stay asynchronous; the per-word clamped
+  // loads (a dependent global round trip per item) are left to unaligned frames only.
   auto stage = [&](int ty, int b) {
     const int ys = P.row_begin + kIntTy * ty - P.pad - 2;
     for (int i = tid; i < kIntSrcRows * kIntSrcWords; i += kIntTx * kIntTy) {
       const int r = i / kIntSrcWords, q = i - r * kIntSrcWords;
       const int yy = clampi(ys + r, 0, P.H - 1);
       uint32_t* d = &tile[b][r * kIntStride + q];
-      if (fast) int_cp4(d, reinterpret_cast<const uint32_t*>(P.rf + (size_t)yy * P.W + xs) + q);
-      else *d = load4_clamped(P.rf, P.W, P.H, xs + 4 * q, yy);
+      if (fast) {
+        int_cp4(d, reinterpret_cast<const uint32_t*>(P.rf + (size_t)yy * P.W + xs) + q);
+      } else if (P.vec_ok) {
+        const int x = min(max(xs + 4 * q, 0), P.W - 4);      // the edge word for outside words
+        int_cp4(d, P.rf + (size_t)yy * P.W + x);
+      } else {
+        *d = load4_clamped(P.rf, P.W, P.H, xs + 4 * q, yy);
+      }
     }
     asm volatile("cp.async.commit_group;" ::: "memory");
+  };
+  // after this thread's copies of buffer b landed: outside words = their edge byte x 4
+  auto edge_fix = [&](int b) {
+    if (fast || !P.vec_ok) return;
+    for (int i = tid; i < kIntSrcRows * kIntSrcWords; i += kIntTx * kIntTy) {
+      const int r = i / kIntSrcWords, q = i - r * kIntSrcWords;
+      const int x = xs + 4 * q;
+      uint32_t* d = &tile[b][r * kIntStride + q];
+      if (x < 0) *d = 0x01010101u * (*d & 0xffu);                 // column 0
+      else if (x + 4 > P.W) *d = 0x01010101u * (*d >> 24);        // column W - 1
+    }
   };
   const int n_ty = (P.row_end - P.row_begin + kIntTy - 1) / kIntTy;
   const int ty0 = FEVES_INT_TPC * blockIdx.y, ty1 = min(n_ty, ty0 + FEVES_INT_TPC);
@@ -259,6 +284,7 @@ __global__ void __launch_bounds__(kIntTx * kIntTy) int_tile_kernel(const IntPara
     } else {
       asm volatile("cp.async.wait_group 0;" ::: "memory");
     }
+    edge_fix(b);
     __syncthreads();
     const int g = g0 + threadIdx.x, rr = P.row_begin + kIntTy * ty + threadIdx.y;
     if (g < groups && rr < P.row_end) {
