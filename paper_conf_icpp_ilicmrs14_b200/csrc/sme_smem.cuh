@@ -33,6 +33,9 @@ namespace feves {
 #ifndef FEVES_SME2_REGION   // staged bytes per CTA (4 planes); larger boxes -> overflow list
 #define FEVES_SME2_REGION (FEVES_SME2_MB == 4 ? 32 * 1024 : 68 * 1024)
 #endif
+#ifndef FEVES_SME2_PITCH    // staged row pitch alignment in bytes (128: vertical MV differences keep the banks)
+#define FEVES_SME2_PITCH 16
+#endif
 #ifndef FEVES_SME2_MINB
 #define FEVES_SME2_MINB (FEVES_SME2_MB == 4 ? 6 : 3)
 #endif
@@ -316,7 +319,8 @@ __global__ void __launch_bounds__(kSme2Threads, FEVES_SME2_MINB) sme_smem_kernel
   __syncthreads();
   xlo = box4[0]; xhi = box4[1]; ylo = box4[2]; yhi = box4[3];
   const int X0 = (xlo + P.pad) & ~15, X1 = (xhi + P.pad + 15) & ~15;   // plane columns, 16-byte aligned
-  const int WB = X1 - X0, RH = yhi - ylo;
+  const int CW = X1 - X0, RH = yhi - ylo;                    // copied bytes per row
+  const int WB = (CW + FEVES_SME2_PITCH - 1) & ~(FEVES_SME2_PITCH - 1);   // staged row pitch
   if (4 * WB * RH > FEVES_SME2_REGION) {                   // does not fit: global-load code afterwards
     if (tid == 0) {
       const int k = atomicAdd(ovf, 1);
@@ -327,13 +331,13 @@ __global__ void __launch_bounds__(kSme2Threads, FEVES_SME2_MINB) sme_smem_kernel
   // ---- stage 4 planes (G, b, h, j) x RH rows x WB bytes: one TMA bulk copy per row (one
   // thread each, completing on the mbarrier), and the CF rows through registers ----
   {
-    if (tid == 0) mbar_expect_tx(bar, (uint32_t)(4 * WB * RH));
+    if (tid == 0) mbar_expect_tx(bar, (uint32_t)(4 * CW * RH));
     int k = 0, rr = tid;                                   // row tid of the 4 * RH (plane, row) pairs
     while (rr >= RH && k < 4) { rr -= RH; ++k; }
     for (; k < 4;) {
       const int ph = (k & 1) * 2 + (k >> 1) * 8;          // plane index: 0 G, 2 b, 8 h, 10 j
       bulk_g2s(s_reg + (uint32_t)((k * RH + rr) * WB),
-               sf + (size_t)ph * P.plane + (size_t)(ylo + rr + P.pad) * P.pitch + X0, (uint32_t)WB, bar);
+               sf + (size_t)ph * P.plane + (size_t)(ylo + rr + P.pad) * P.pitch + X0, (uint32_t)CW, bar);
       rr += kSme2Threads;
       while (rr >= RH && k < 4) { rr -= RH; ++k; }
     }
