@@ -97,7 +97,6 @@ struct me_ctx {
   int graph;             // ME_OPT_GRAPH
   int sme_kernel;        // ME_OPT_SME_KERNEL: 0 global-load SME (default), 1 shared-memory staged
   int int_kernel;        // ME_OPT_INT_KERNEL: 0 per-thread global loads, 1 shared-memory tiled
-  int me_ws;             // ME_OPT_ME_WS: warp-specialised S = 64 ME kernel (me_ws.cuh)
   // me_stream_push_flags: stream-ordered peer flags of the push being enqueued
   const uint32_t* wait_flag; uint32_t wait_value;     // the frame copy waits for *wait_flag >= wait_value
   uint32_t* signal_flag; uint32_t signal_value;       // written once the push's outputs are complete
@@ -141,7 +140,6 @@ static cudaError_t set_me_smem(int bytes) {
   if (e == cudaSuccess) e = me_set_smem_32(bytes);
   if (e == cudaSuccess) e = me_set_smem_64(bytes);
   if (e == cudaSuccess) e = me_set_smem_128(bytes);
-  if (e == cudaSuccess) e = me_ws_init_64();
   return e;
 }
 
@@ -320,7 +318,6 @@ extern "C" me_ctx* me_create_pmv(int width, int height, int sa_range, int n_rf, 
   if (ok) {
     c->stream = c->own;
     c->int_kernel = 1;   // shared-memory tiled INT: 11.2 vs 14.2 us (ncu, 1080p S64)
-    c->me_ws = 0;   // warp-specialised S = 64 kernel: measured slower (0.97-1.03 vs 0.83 ms), DESIGN.md §6
     c->sme_kernel = 0;   // the staged SME measured on par (145-149 vs 145 us at 1080p S64 4 RF): opt-in
     ok = upload_key_table(c) == ME_OK && sme2_init() == cudaSuccess &&
          set_me_smem(200 * 1024) == cudaSuccess;   // max; the launch asks for what it needs
@@ -475,13 +472,6 @@ static int launch_me(me_ctx* c, const uint8_t* cf, const uint8_t* const* rfs, in
                     : c->max_pmv ? (c->lambda ? kMePmvRate : kMePmv)
                     : c->lambda ? kMeRate : kMePlain;
   cudaError_t e;
-  if (c->me_ws && c->S == 64 && variant == kMePlain && !c->inclusive && c->me_ctas_per_sm == 0) {
-    e = me_ws_launch_64(grid, st, P);   // warp-specialised (me_ws.cuh)
-    if (e != cudaSuccess) { fprintf(stderr, "feves_me: ME launch: %s\n", cudaGetErrorString(e)); return ME_ECUDA; }
-    tmark(c, 3, st);
-    c->last_launches++;
-    return launch_status();
-  }
   switch (c->inclusive || (c->max_pmv && c->S == 128) ? 0 : c->S) {   // compile-time window geometry for the paper's SA sizes (Fig. 6a: 32..256)
     case 16: e = me_launch_16(variant, grid, c->me_threads, smem, st, P); break;
     case 32: e = me_launch_32(variant, grid, c->me_threads, smem, st, P); break;
@@ -1086,10 +1076,6 @@ extern "C" int me_set_option(me_ctx* c, int option, int value) {
     case ME_OPT_INT_KERNEL:
       if (value < 0 || value > 1) return ME_EINVAL;
       c->int_kernel = value;
-      return ME_OK;
-    case ME_OPT_ME_WS:
-      if (value < 0 || value > 1) return ME_EINVAL;
-      c->me_ws = value;
       return ME_OK;
     case ME_OPT_SME_KERNEL:
       if (value < 0 || value > 1) return ME_EINVAL;

@@ -66,11 +66,6 @@ FEVES_ME_TU_DECL(128)
   }                                                                                                   \
   cudaError_t me_set_smem_##SS(int bytes) { return me_set_smem_tmpl<SS>(bytes); }
 
-// warp-specialised ME for S = 64, base reading (me_ws.cuh; defined in me_s64.cu)
-cudaError_t me_ws_launch_64(dim3 grid, cudaStream_t st, const MeParams& P);
-cudaError_t me_ws_init_64();   // dynamic shared-memory attribute
-size_t me_ws_smem_bytes_64();
-
 // SME (sme.cu): rd = rate term compiled in (G18), satd = Hadamard distortion (G20)
 cudaError_t sme_launch(bool rd, bool satd, dim3 grid, int threads, cudaStream_t st, const SmeParams& P);
 // SME with shared-memory staged windows (sme_smem.cuh), one CTA per group of 8 MBs x RF:
