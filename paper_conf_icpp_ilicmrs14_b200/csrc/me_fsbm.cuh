@@ -74,7 +74,10 @@ __host__ __device__ constexpr int me_nsub(int S) { return 32 / me_lx(S); }
 #ifndef FEVES_ME_NWY64
 #define FEVES_ME_NWY64 1
 #endif
-__host__ __device__ constexpr int me_nwy(int S) { return S == 16 ? 2 : S == 64 ? FEVES_ME_NWY64 : 1; }
+#ifndef FEVES_ME_NWY32
+#define FEVES_ME_NWY32 1
+#endif
+__host__ __device__ constexpr int me_nwy(int S) { return S == 16 ? 2 : S == 32 ? FEVES_ME_NWY32 : S == 64 ? FEVES_ME_NWY64 : 1; }
 __host__ __device__ constexpr int me_dyl(int S) {
   return ((S + me_nsub(S) * me_nwy(S) - 1) / (me_nsub(S) * me_nwy(S)) + kMeT - 1) / kMeT * kMeT;
 }
