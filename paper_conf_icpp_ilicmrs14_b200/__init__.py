@@ -308,7 +308,8 @@ class MotionEstimator:
         _check(lib().me_set_fused(self._ctx, int(on)))
 
     OPT_FUSED_SME, OPT_PIPELINE_RF, OPT_ME_CTAS_PER_SM, OPT_LAMBDA, OPT_SME_SATD, OPT_SA_INCLUSIVE = 1, 2, 3, 4, 5, 6
-    OPT_HALO_ONLY, OPT_OVERLAP_SME, OPT_GRAPH, OPT_SME_KERNEL, OPT_INT_KERNEL = 7, 8, 9, 10, 11
+    OPT_HALO_ONLY, OPT_OVERLAP_SME, OPT_GRAPH, OPT_SME_KERNEL, OPT_INT_KERNEL, OPT_RF_PER_CTA = 7, 8, 9, 10, 11, 12
+    OPT_SME_SPLIT = 13
 
     def set_sa_inclusive(self, on: bool = True):
         """Candidates in [-S/2, +S/2]^2 (G1 alternative reading, f4)."""

@@ -97,6 +97,9 @@ struct me_ctx {
   int graph;             // ME_OPT_GRAPH
   int sme_kernel;        // ME_OPT_SME_KERNEL: 0 global-load SME (default), 1 shared-memory staged
   int int_kernel;        // ME_OPT_INT_KERNEL: 0 per-thread global loads, 1 shared-memory tiled
+  int rf_per_cta;        // ME_OPT_RF_PER_CTA: RFs per ME CTA (0 = all)
+  int sme_split;         // ME_OPT_SME_SPLIT: 0 auto, 1 never, 2 always (one partition group per SME warp)
+  int sme_split_warps;   // auto: split below this many mode-warps
   // me_stream_push_flags: stream-ordered peer flags of the push being enqueued
   const uint32_t* wait_flag; uint32_t wait_value;     // the frame copy waits for *wait_flag >= wait_value
   uint32_t* signal_flag; uint32_t signal_value;       // written once the push's outputs are complete
@@ -318,6 +321,9 @@ extern "C" me_ctx* me_create_pmv(int width, int height, int sa_range, int n_rf, 
   if (ok) {
     c->stream = c->own;
     c->int_kernel = 1;   // shared-memory tiled INT: 11.2 vs 14.2 us (ncu, 1080p S64)
+    c->sme_split = 0;
+    c->sme_split_warps = 6 * 148 * 20;   // ~ six waves of the SME kernel (20 resident warps/SM): 1080p on 2+ GPUs
+    c->rf_per_cta = 1;   // one CTA per (MB, RF): 1080p S64 4 RF ME 820.6 vs 837.1 us, 9-row stripe 124.1 vs 144.8 us
     c->sme_kernel = 0;   // the staged SME measured on par (145-149 vs 145 us at 1080p S64 4 RF): opt-in
     ok = upload_key_table(c) == ME_OK && sme2_init() == cudaSuccess &&
          set_me_smem(200 * 1024) == cudaSuccess;   // max; the launch asks for what it needs
@@ -463,7 +469,13 @@ static int launch_me(me_ctx* c, const uint8_t* cf, const uint8_t* const* rfs, in
     P.out_qmvs = reinterpret_cast<uint32_t*>(qmvs);
     P.out_qsads = qsads;
   }
-  dim3 grid(c->mb_cols, c->row1 - c->row0);
+  // RFs per CTA (ME_OPT_RF_PER_CTA, default 1: one CTA per (MB, RF)): more, shorter CTAs
+  // desynchronise their window stagings across waves and shorten the last wave -- the frame and,
+  // more so, a narrow MB-row stripe of a multi-GPU split
+  int rpc = n_ref;
+  if (!fused && c->rf_per_cta > 0) rpc = std::min(n_ref, c->rf_per_cta);
+  P.rf_per_cta = rpc;
+  dim3 grid(c->mb_cols, c->row1 - c->row0, (n_ref + rpc - 1) / rpc);
   size_t smem = fused ? c->me_smem_fused : c->me_smem;
   if (c->me_ctas_per_sm > 0)   // occupancy cap: leave registers / warps for a co-running SME
     smem = std::max(smem, (size_t)(228 * 1024) / (size_t)(c->me_ctas_per_sm + 1) - 1024 + 64);
@@ -550,6 +562,10 @@ static int launch_sme(me_ctx* c, const uint8_t* cf, const uint8_t* const* sfs, c
   P.cf_vec = (c->W % 4 == 0) && ((reinterpret_cast<uintptr_t>(cf) & 3) == 0);   // aligned CF word loads
   P.k_hi = kAvgHi;
   const int warps = n_ref * P.n_rows * P.groups;
+  // one partition group per warp (16 tasks per MB group instead of 7 modes) when the grid would
+  // not fill the GPU ~6 times over (ME_OPT_SME_SPLIT: 0 auto, 1 never, 2 always; 1080p: split on
+  // 2+ GPUs, 34-row stripe SME 78.8 vs 83.5 us, 9-row 32.8 vs 44.2 us; whole frame 153.1 vs 148.4 us)
+  P.split = c->sme_split == 2 || (c->sme_split == 0 && 7 * warps < c->sme_split_warps);
   if (marks & 1) tmark(c, 4, st);
   // shared-memory staged SME (sme_smem.cuh) for the SAD distortion with the ME SADs given
   // and 16-byte aligned SFs (cp.async); the global-load kernel otherwise
@@ -560,7 +576,7 @@ static int launch_sme(me_ctx* c, const uint8_t* cf, const uint8_t* const* sfs, c
     e = sme2_launch(c->lambda != 0, n_ref * P.n_rows * ((c->mb_cols + kSme2Mb - 1) / kSme2Mb), st, P, c->d_ovf);
     c->last_launches += 2;
   } else {
-    const dim3 sg((warps + 3) / 4, 7);   // y = partition mode
+    const dim3 sg((warps + 3) / 4, P.split ? 16 : 7);   // y = partition mode (or mode x group)
     e = sme_launch(c->lambda != 0, c->satd != 0, sg, 128, st, P);
     c->last_launches++;
   }
@@ -1076,6 +1092,14 @@ extern "C" int me_set_option(me_ctx* c, int option, int value) {
     case ME_OPT_INT_KERNEL:
       if (value < 0 || value > 1) return ME_EINVAL;
       c->int_kernel = value;
+      return ME_OK;
+    case ME_OPT_SME_SPLIT:
+      if (value < 0 || value > 2) return ME_EINVAL;
+      c->sme_split = value;
+      return ME_OK;
+    case ME_OPT_RF_PER_CTA:
+      if (value < 0 || value > kMaxRf) return ME_EINVAL;
+      c->rf_per_cta = value;
       return ME_OK;
     case ME_OPT_SME_KERNEL:
       if (value < 0 || value > 1) return ME_EINVAL;

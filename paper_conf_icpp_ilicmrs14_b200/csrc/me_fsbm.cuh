@@ -56,6 +56,7 @@ struct MeParams {
   const int16_t* pmv;         // G21 predictor [frame MB][rf_stride][2] integer-pel (runtime-S kernel only), or null
   int max_pmv;                // G21 clamp of each predictor component
   int vec_ok;                 // 16-byte aligned rows and window start: vector staging allowed
+  int rf_per_cta;             // RFs searched per CTA: CTA (x, y, z) takes RFs [z * rf_per_cta, +rf_per_cta)
   // fused SME (template FUSE): SF of each RF, quarter-pel outputs
   const uint8_t* sf[kMaxRf];
   int sf_pad, sf_pitch;
@@ -419,7 +420,8 @@ __global__ void __launch_bounds__(S_CT ? 128 : 256, S_CT ? FEVES_ME_MINB : 2) me
   constexpr int NSTG = S_CT ? me_nstage(S_CT) : 1;      // window stagings per RF (dy halves)
   const int win_rows = S_CT ? me_win_rows(S_CT) : S + 15;
 
-  for (int ref = 0; ref < P.n_rf; ++ref) {
+  const int ref_begin = (int)blockIdx.z * P.rf_per_cta, ref_end = min(P.n_rf, ref_begin + P.rf_per_cta);
+  for (int ref = ref_begin; ref < ref_end; ++ref) {
     const uint8_t* __restrict__ rf = P.rf[ref];
     // G21: the SA of this (MB, RF) is centred on the clamped predictor p (runtime-S kernel and the
     // PMV instantiations; the default compile-time kernels never see a predictor, code unchanged)
@@ -495,7 +497,7 @@ __global__ void __launch_bounds__(S_CT ? 128 : 256, S_CT ? FEVES_ME_MINB : 2) me
                        __byte_perm(w[2], w[3], 0x6543), __byte_perm(w[3], w[4], 0x6543));
       }
     }
-    if (kLateCf && ref == 0) {
+    if (kLateCf && ref == ref_begin) {                   // the CTA's first RF
 #pragma unroll
       for (int j = 0; j < 2; ++j) {
         const int i = threadIdx.x + j * (int)blockDim.x;

@@ -40,6 +40,7 @@ struct SmeParams {
   int fence;                                          // outputs are peer memory (me_ipc_open): system fence at exit
   int cf_vec;                                         // W % 4 == 0 and cf 4-byte aligned: CF rows as aligned words
   uint32_t k_hi;                                      // = kAvgHi (vavg4)
+  int split;                                          // grid.y = 16 (mode, partition group) tasks instead of 7 modes
 };
 
 // ring-1 spiral order s_k (G12/G14), compile-time so unrolled loops fold it
@@ -298,18 +299,19 @@ __device__ __forceinline__ int mode_part(int bx, int by) {
 // RD = rate term (G18) compiled in; SATD = Hadamard distortion (G20) instead of SAD
 template <int MODE, int YG, int XMASK, bool RD, bool SATD>
 __device__ __forceinline__ void refine_mode(const SmeParams& P, const uint8_t* __restrict__ sf, size_t o, int bx,
-                                            int xs, int ys0, bool writer, int qpx, int qpy) {
+                                            int xs, int ys0, bool writer, int qpx, int qpy, int g0 = 0, int g1 = 4) {
   constexpr int NG = 4 / YG;           // partitions (block groups) inside this lane's strip
+  g1 = min(g1, NG);                    // this warp refines groups [g0, g1) (all NG, or one: P.split)
   // The groups are refined one after the other (latency-bound kernel: fewer live
   // registers -> more resident warps beats the ILP of refining all NG at once).
   // the next group's ME result (MV, SAD) is loaded one group ahead, so only the first
   // group pays the dependent MV -> SF-address round trip
-  uint32_t mv_n = __ldg(P.in_mvs + o + mode_part<MODE>(bx, 0));
-  uint32_t sad_n = (P.in_sads && !SATD) ? (uint32_t)__ldg(P.in_sads + o + mode_part<MODE>(bx, 0)) : 0u;
+  uint32_t mv_n = __ldg(P.in_mvs + o + mode_part<MODE>(bx, g0 * YG));
+  uint32_t sad_n = (P.in_sads && !SATD) ? (uint32_t)__ldg(P.in_sads + o + mode_part<MODE>(bx, g0 * YG)) : 0u;
 #pragma unroll 1
-  for (int g = 0; g < NG; ++g) {
+  for (int g = g0; g < g1; ++g) {
     const uint32_t mv = mv_n, sad_me = sad_n;
-    if (g + 1 < NG) {
+    if (g + 1 < g1) {
       const int pn = mode_part<MODE>(bx, (g + 1) * YG);
       mv_n = __ldg(P.in_mvs + o + pn);
       if (P.in_sads && !SATD) sad_n = __ldg(P.in_sads + o + pn);
@@ -451,14 +453,24 @@ __global__ void __launch_bounds__(128, FEVES_SME_MINB) sme_refine_kernel(const S
     qpx = 4 * min(max((int)P.pmv[2 * pi], -P.max_pmv), P.max_pmv);
     qpy = 4 * min(max((int)P.pmv[2 * pi + 1], -P.max_pmv), P.max_pmv);
   }
-  switch (blockIdx.y) {   // one mode per warp: 7x the independent warps (the kernel is latency-bound)
-    case 0: refine_mode<0, 4, 3, RD, SATD>(P, sf, o, bx, xs, ys0, writer, qpx, qpy); break;   // 16x16
-    case 1: refine_mode<1, 2, 3, RD, SATD>(P, sf, o, bx, xs, ys0, writer, qpx, qpy); break;   // 16x8
-    case 2: refine_mode<2, 4, 1, RD, SATD>(P, sf, o, bx, xs, ys0, writer, qpx, qpy); break;   // 8x16
-    case 3: refine_mode<3, 2, 1, RD, SATD>(P, sf, o, bx, xs, ys0, writer, qpx, qpy); break;   // 8x8
-    case 4: refine_mode<4, 1, 1, RD, SATD>(P, sf, o, bx, xs, ys0, writer, qpx, qpy); break;   // 8x4
-    case 5: refine_mode<5, 2, 0, RD, SATD>(P, sf, o, bx, xs, ys0, writer, qpx, qpy); break;   // 4x8
-    default: refine_mode<6, 1, 0, RD, SATD>(P, sf, o, bx, xs, ys0, writer, qpx, qpy); break;  // 4x4
+  // one mode per warp: 7x the independent warps (the kernel is latency-bound); with P.split one
+  // partition group per warp (16 tasks: modes with 1, 2, 1, 2, 4, 2, 4 groups), for grids too small
+  // to fill the GPU with 7 (a narrow MB-row stripe)
+  int mode = blockIdx.y, g0 = 0, g1 = 4;
+  if (P.split) {
+    const int y = blockIdx.y;
+    mode = y < 1 ? 0 : y < 3 ? 1 : y < 4 ? 2 : y < 6 ? 3 : y < 10 ? 4 : y < 12 ? 5 : 6;
+    g0 = y - (mode == 0 ? 0 : mode == 1 ? 1 : mode == 2 ? 3 : mode == 3 ? 4 : mode == 4 ? 6 : mode == 5 ? 10 : 12);
+    g1 = g0 + 1;
+  }
+  switch (mode) {
+    case 0: refine_mode<0, 4, 3, RD, SATD>(P, sf, o, bx, xs, ys0, writer, qpx, qpy, g0, g1); break;   // 16x16
+    case 1: refine_mode<1, 2, 3, RD, SATD>(P, sf, o, bx, xs, ys0, writer, qpx, qpy, g0, g1); break;   // 16x8
+    case 2: refine_mode<2, 4, 1, RD, SATD>(P, sf, o, bx, xs, ys0, writer, qpx, qpy, g0, g1); break;   // 8x16
+    case 3: refine_mode<3, 2, 1, RD, SATD>(P, sf, o, bx, xs, ys0, writer, qpx, qpy, g0, g1); break;   // 8x8
+    case 4: refine_mode<4, 1, 1, RD, SATD>(P, sf, o, bx, xs, ys0, writer, qpx, qpy, g0, g1); break;   // 8x4
+    case 5: refine_mode<5, 2, 0, RD, SATD>(P, sf, o, bx, xs, ys0, writer, qpx, qpy, g0, g1); break;   // 4x8
+    default: refine_mode<6, 1, 0, RD, SATD>(P, sf, o, bx, xs, ys0, writer, qpx, qpy, g0, g1); break;  // 4x4
   }
   if (P.fence) __threadfence_system();   // stores to another GPU's buffer are performed before the kernel ends
 }

@@ -280,3 +280,23 @@ def test_set_stream_own_stream_kept(feves, orc):
     np.testing.assert_array_equal(s.cpu().numpy().reshape(n, 1, 41), o_s)
     np.testing.assert_array_equal(m.cpu().numpy().reshape(n, 1, 41, 2), o_m)
     me.close()
+
+
+@pytest.mark.parametrize("S", [16, 32, 64, 12])
+@pytest.mark.parametrize("rpc", [0, 1, 2])
+def test_rf_per_cta_split(feves, orc, S, rpc):
+    """ME_OPT_RF_PER_CTA: the RFs of an MB spread over grid.z CTAs (1 or 2 RFs each, 0 = all in
+    one CTA) give the oracle's result for every RF -- compile-time S (incl. the S <= 32 late CF
+    store of each CTA's first RF) and the run-time-S kernel (S = 12), 3 RFs, ragged frame"""
+    W, H = 72, 40
+    frames = [gen_tex(W, H, t, 21 + S) for t in range(4)]
+    cf, rfs = frames[3], [frames[2], frames[1], frames[0]]
+    me = feves.MotionEstimator(W, H, S, 3)
+    me.set_option(me.OPT_RF_PER_CTA, rpc)
+    m, s = me.estimate(_dev(cf), [_dev(r) for r in rfs])
+    torch.cuda.synchronize()
+    n = me.mb_rows * me.mb_cols
+    o_m, o_s = orc.me(cf, rfs, S)
+    np.testing.assert_array_equal(s.cpu().numpy().reshape(n, 3, 41), o_s)
+    np.testing.assert_array_equal(m.cpu().numpy().reshape(n, 3, 41, 2), o_m)
+    me.close()
