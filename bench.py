@@ -54,6 +54,8 @@ def parse():
                          "(auto: full when the calibrated estimate is <= --cpu-full-max seconds)")
     ap.add_argument("--cpu-full-max", type=float, default=90.0)
     ap.add_argument("--sme-kernel", type=int, default=None, help="ME_OPT_SME_KERNEL (0 global-load, 1 staged)")
+    ap.add_argument("--rf-per-cta", type=int, default=None, help="ME_OPT_RF_PER_CTA (0 = all RFs in one CTA)")
+    ap.add_argument("--sme-split", type=int, default=None, help="ME_OPT_SME_SPLIT (0 auto, 1 never, 2 always)")
     ap.add_argument("--graph", type=int, default=1,
                     help="ME_OPT_GRAPH: one CUDA graph per frame (default 1; 0 = multi-stream enqueue)")
     ap.add_argument("--pipeline", type=int, default=None, help="ME_OPT_PIPELINE_RF (default: library default)")
@@ -450,7 +452,8 @@ def run_feves(args, cfg):
     me.set_rows(r0, r1)      # (ShardedStream may re-split later in adaptive mode)
     for opt, val in ((me.OPT_PIPELINE_RF, args.pipeline), (me.OPT_ME_CTAS_PER_SM, args.me_ctas),
                      (me.OPT_FUSED_SME, args.fused), (me.OPT_GRAPH, args.graph if world == 1 else None),
-                     (me.OPT_SME_KERNEL, args.sme_kernel)):
+                     (me.OPT_SME_KERNEL, args.sme_kernel), (me.OPT_RF_PER_CTA, args.rf_per_cta),
+                     (me.OPT_SME_SPLIT, args.sme_split)):
         if val is not None:
             me.set_option(opt, val)
     me.set_timing(False)                 # as in the timed pass: the graphs captured during the fill are its own

@@ -97,7 +97,7 @@ struct me_ctx {
   int graph;             // ME_OPT_GRAPH
   int sme_kernel;        // ME_OPT_SME_KERNEL: 0 global-load SME (default), 1 shared-memory staged
   int int_kernel;        // ME_OPT_INT_KERNEL: 0 per-thread global loads, 1 shared-memory tiled
-  int rf_per_cta;        // ME_OPT_RF_PER_CTA: RFs per ME CTA (0 = all)
+  int rf_per_cta;        // ME_OPT_RF_PER_CTA: RFs per ME CTA (0 = all, -1 = auto)
   int sme_split;         // ME_OPT_SME_SPLIT: 0 auto, 1 never, 2 always (one partition group per SME warp)
   int sme_split_warps;   // auto: split below this many mode-warps
   // me_stream_push_flags: stream-ordered peer flags of the push being enqueued
@@ -323,7 +323,8 @@ extern "C" me_ctx* me_create_pmv(int width, int height, int sa_range, int n_rf, 
     c->int_kernel = 1;   // shared-memory tiled INT: 11.2 vs 14.2 us (ncu, 1080p S64)
     c->sme_split = 0;
     c->sme_split_warps = 6 * 148 * 20;   // ~ six waves of the SME kernel (20 resident warps/SM): 1080p on 2+ GPUs
-    c->rf_per_cta = 1;   // one CTA per (MB, RF): 1080p S64 4 RF ME 820.6 vs 837.1 us, 9-row stripe 124.1 vs 144.8 us
+    c->rf_per_cta = -1;  // auto: one CTA per (MB, RF) (1080p S64 4 RF ME 818.5 vs 834.5 us, 9-row stripe
+                         // 124.1 vs 144.8 us); 2 RFs per CTA at S = 128 (2160p ME 12.50 vs 12.62 ms)
     c->sme_kernel = 0;   // the staged SME measured on par (145-149 vs 145 us at 1080p S64 4 RF): opt-in
     ok = upload_key_table(c) == ME_OK && sme2_init() == cudaSuccess &&
          set_me_smem(200 * 1024) == cudaSuccess;   // max; the launch asks for what it needs
@@ -473,7 +474,8 @@ static int launch_me(me_ctx* c, const uint8_t* cf, const uint8_t* const* rfs, in
   // desynchronise their window stagings across waves and shorten the last wave -- the frame and,
   // more so, a narrow MB-row stripe of a multi-GPU split
   int rpc = n_ref;
-  if (!fused && c->rf_per_cta > 0) rpc = std::min(n_ref, c->rf_per_cta);
+  const int want = c->rf_per_cta < 0 ? (c->S >= 128 ? 2 : 1) : c->rf_per_cta;
+  if (!fused && want > 0) rpc = std::min(n_ref, want);
   P.rf_per_cta = rpc;
   dim3 grid(c->mb_cols, c->row1 - c->row0, (n_ref + rpc - 1) / rpc);
   size_t smem = fused ? c->me_smem_fused : c->me_smem;
@@ -1098,7 +1100,7 @@ extern "C" int me_set_option(me_ctx* c, int option, int value) {
       c->sme_split = value;
       return ME_OK;
     case ME_OPT_RF_PER_CTA:
-      if (value < 0 || value > kMaxRf) return ME_EINVAL;
+      if (value < -1 || value > kMaxRf) return ME_EINVAL;
       c->rf_per_cta = value;
       return ME_OK;
     case ME_OPT_SME_KERNEL:

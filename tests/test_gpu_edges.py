@@ -282,12 +282,13 @@ def test_set_stream_own_stream_kept(feves, orc):
     me.close()
 
 
-@pytest.mark.parametrize("S", [16, 32, 64, 12])
-@pytest.mark.parametrize("rpc", [0, 1, 2])
+@pytest.mark.parametrize("S", [16, 32, 64, 128, 12])
+@pytest.mark.parametrize("rpc", [-1, 0, 1, 2])
 def test_rf_per_cta_split(feves, orc, S, rpc):
     """ME_OPT_RF_PER_CTA: the RFs of an MB spread over grid.z CTAs (1 or 2 RFs each, 0 = all in
-    one CTA) give the oracle's result for every RF -- compile-time S (incl. the S <= 32 late CF
-    store of each CTA's first RF) and the run-time-S kernel (S = 12), 3 RFs, ragged frame"""
+    one CTA, -1 auto) give the oracle's result for every RF -- compile-time S (incl. the S <= 32 late CF
+    store of each CTA's first RF, the S = 128 quadrant keys) and the run-time-S kernel (S = 12), 3 RFs,
+    ragged frame"""
     W, H = 72, 40
     frames = [gen_tex(W, H, t, 21 + S) for t in range(4)]
     cf, rfs = frames[3], [frames[2], frames[1], frames[0]]
