@@ -564,10 +564,12 @@ static int launch_sme(me_ctx* c, const uint8_t* cf, const uint8_t* const* sfs, c
   P.cf_vec = (c->W % 4 == 0) && ((reinterpret_cast<uintptr_t>(cf) & 3) == 0);   // aligned CF word loads
   P.k_hi = kAvgHi;
   const int warps = n_ref * P.n_rows * P.groups;
-  // one partition group per warp (16 tasks per MB group instead of 7 modes) when the grid would
-  // not fill the GPU ~6 times over (ME_OPT_SME_SPLIT: 0 auto, 1 never, 2 always; 1080p: split on
-  // 2+ GPUs, 34-row stripe SME 78.8 vs 83.5 us, 9-row 32.8 vs 44.2 us; whole frame 153.1 vs 148.4 us)
-  P.split = c->sme_split == 2 || (c->sme_split == 0 && 7 * warps < c->sme_split_warps);
+  // SME work per warp (ME_OPT_SME_SPLIT): 1 = one mode (7 warps per MB group, all its partition
+  // groups in turn), 2 = one partition group (16 warps), 3 = the 4-group modes as two warps of two
+  // groups (9 warps); 0 (auto) = 3 when the grid would not fill the GPU ~6 times over, else 1.
+  // 1080p S64 4 RF (tools/stripe_probe.py): whole frame 141.2 (1) / 143.4 (3) / 153.1 us (2);
+  // 34-row stripe 80.9 (2) / 75.8 us (3); 9-row stripe 44.2 (1) / 33.8 (2) / 31.6 us (3)
+  P.split = (c->sme_split == 3 || (c->sme_split == 0 && 7 * warps < c->sme_split_warps)) ? 3 : c->sme_split == 2 ? 1 : 0;
   if (marks & 1) tmark(c, 4, st);
   // shared-memory staged SME (sme_smem.cuh) for the SAD distortion with the ME SADs given
   // and 16-byte aligned SFs (cp.async); the global-load kernel otherwise
@@ -578,7 +580,7 @@ static int launch_sme(me_ctx* c, const uint8_t* cf, const uint8_t* const* sfs, c
     e = sme2_launch(c->lambda != 0, n_ref * P.n_rows * ((c->mb_cols + kSme2Mb - 1) / kSme2Mb), st, P, c->d_ovf);
     c->last_launches += 2;
   } else {
-    const dim3 sg((warps + 3) / 4, P.split ? 16 : 7);   // y = partition mode (or mode x group)
+    const dim3 sg((warps + 3) / 4, P.split == 3 ? 9 : P.split ? 16 : 7);   // y = partition mode (or mode x groups)
     e = sme_launch(c->lambda != 0, c->satd != 0, sg, 128, st, P);
     c->last_launches++;
   }
@@ -1096,7 +1098,7 @@ extern "C" int me_set_option(me_ctx* c, int option, int value) {
       c->int_kernel = value;
       return ME_OK;
     case ME_OPT_SME_SPLIT:
-      if (value < 0 || value > 2) return ME_EINVAL;
+      if (value < 0 || value > 3) return ME_EINVAL;
       c->sme_split = value;
       return ME_OK;
     case ME_OPT_RF_PER_CTA:

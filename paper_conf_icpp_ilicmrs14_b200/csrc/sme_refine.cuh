@@ -456,8 +456,18 @@ __global__ void __launch_bounds__(128, FEVES_SME_MINB) sme_refine_kernel(const S
   // one mode per warp: 7x the independent warps (the kernel is latency-bound); with P.split one
   // partition group per warp (16 tasks: modes with 1, 2, 1, 2, 4, 2, 4 groups), for grids too small
   // to fill the GPU with 7 (a narrow MB-row stripe)
-  int mode = blockIdx.y, g0 = 0, g1 = 4;
-  if (P.split) {
+#ifndef FEVES_SME_LPT
+#define FEVES_SME_LPT 1   // measured 140.4 vs 146.8 us at 1080p S64 4 RF (the long warps no longer form the tail)
+#endif
+  // FEVES_SME_LPT: the modes with the most partition groups per warp (4x4, 8x4: four dependent
+  // MV -> sweep chains) are dispatched first, the single-group modes last
+  int mode = FEVES_SME_LPT ? (0x0213546 >> (4 * (int)blockIdx.y)) & 15 : (int)blockIdx.y, g0 = 0, g1 = 4;
+  if (P.split == 3) {                 // 9 tasks: the 4-group modes as two warps of 2 groups, longest first
+    const int y = blockIdx.y;         // (6: 0-1), (6: 2-3), (4: 0-1), (4: 2-3), 5, 3, 1, 2, 0
+    mode = y < 2 ? 6 : y < 4 ? 4 : (0x021350000 >> (4 * y)) & 15;
+    g0 = y < 4 ? 2 * (y & 1) : 0;
+    g1 = y < 4 ? g0 + 2 : 4;
+  } else if (P.split) {
     const int y = blockIdx.y;
     mode = y < 1 ? 0 : y < 3 ? 1 : y < 4 ? 2 : y < 6 ? 3 : y < 10 ? 4 : y < 12 ? 5 : 6;
     g0 = y - (mode == 0 ? 0 : mode == 1 ? 1 : mode == 2 ? 3 : mode == 3 ? 4 : mode == 4 ? 6 : mode == 5 ? 10 : 12);

@@ -301,3 +301,24 @@ def test_rf_per_cta_split(feves, orc, S, rpc):
     np.testing.assert_array_equal(s.cpu().numpy().reshape(n, 3, 41), o_s)
     np.testing.assert_array_equal(m.cpu().numpy().reshape(n, 3, 41, 2), o_m)
     me.close()
+
+
+@pytest.mark.parametrize("split", [0, 1, 2, 3])
+def test_sme_split_modes(feves, orc, split):
+    """ME_OPT_SME_SPLIT: every SME work split (one mode, one partition group, or two groups per
+    warp, longest tasks dispatched first) gives the oracle's refinement on every partition"""
+    W, H, S = 88, 56, 16
+    frames = [gen_tex(W, H, t, 5) for t in range(3)]
+    cf, rfs = frames[2], [frames[1], frames[0]]
+    me = feves.MotionEstimator(W, H, S, 2)
+    me.set_option(me.OPT_SME_SPLIT, split)
+    tcf, trfs = _dev(cf), [_dev(r) for r in rfs]
+    sfs = [me.new_sf() for _ in trfs]
+    (m, s), (q, qs) = me.encode_frame(tcf, trfs, sfs, n_int=2, out_me=me.new_mvs())
+    torch.cuda.synchronize()
+    n = me.mb_rows * me.mb_cols
+    o_m, _ = orc.me(cf, rfs, S)
+    o_q, o_qs = orc.sme(cf, rfs, o_m)
+    np.testing.assert_array_equal(qs.cpu().numpy().reshape(n, 2, 41), o_qs)
+    np.testing.assert_array_equal(q.cpu().numpy().reshape(n, 2, 41, 2), o_q)
+    me.close()
