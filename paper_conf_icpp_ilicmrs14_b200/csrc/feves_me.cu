@@ -322,7 +322,9 @@ extern "C" me_ctx* me_create_pmv(int width, int height, int sa_range, int n_rf, 
     c->stream = c->own;
     c->int_kernel = 1;   // shared-memory tiled INT: 11.2 vs 14.2 us (ncu, 1080p S64)
     c->sme_split = 0;
-    c->sme_split_warps = 6 * 148 * 20;   // ~ six waves of the SME kernel (20 resident warps/SM): 1080p on 2+ GPUs
+    int sms = 148;
+    if (cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, c->device) != cudaSuccess) sms = 148;
+    c->sme_split_warps = 6 * sms * 20;   // ~ six waves of the SME kernel (20 resident warps/SM): 1080p on 2+ GPUs
     c->rf_per_cta = -1;  // auto: one CTA per (MB, RF) (1080p S64 4 RF ME 818.5 vs 834.5 us, 9-row stripe
                          // 124.1 vs 144.8 us); 2 RFs per CTA at S = 128 (2160p ME 12.50 vs 12.62 ms)
     c->sme_kernel = 0;   // the staged SME measured on par (145-149 vs 145 us at 1080p S64 4 RF): opt-in
