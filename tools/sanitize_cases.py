@@ -68,4 +68,17 @@ for (W, H, S, n) in [(200, 72, 64, 2), (854, 40, 32, 1), (200, 72, 128, 1), (33,
     me.sync()
     torch.cuda.synchronize()
     me.close()
+# session 3: every ME RF split and every SME work split (small frames: the auto split is 3)
+for (W, H, S, n) in [(96, 80, 64, 3), (64, 48, 16, 2), (48, 40, 128, 3)]:
+    frames = [torch.from_numpy(gen_tex(W, H, t, 4)).cuda() for t in range(n + 1)]
+    me = F.MotionEstimator(W, H, S, n)
+    sfs = [me.new_sf() for _ in range(n)]
+    for rpc in (-1, 0, 1, 2):
+        for split in (0, 1, 2, 3):
+            me.set_option(me.OPT_RF_PER_CTA, rpc)
+            me.set_option(me.OPT_SME_SPLIT, split)
+            me.encode_frame(frames[n], frames[:n], sfs, n_int=n if rpc == -1 and split == 0 else 0,
+                            out_me=me.new_mvs())
+    torch.cuda.synchronize()
+    me.close()
 print("sanitize cases done")
