@@ -747,7 +747,7 @@ def run_feves(args, cfg):
         "roofline_me_only": {"bound": "alu", "kernel": "me_fsbm_kernel<64> (ME alone, isolated, L2 flushed)",
                              "achieved": me_only_px / 1e12, "peak": peak_px / 1e12, "unit": "Tpx-absdiff/s",
                              "frac": me_only_px / peak_px},
-        "roofline_int": {"bound": "hbm", "kernel": "int_subpel_kernel",
+        "roofline_int": {"bound": "hbm", "kernel": "int_tile_kernel (ME_OPT_INT_KERNEL = 1, default)",
                          "traffic_unit": "16 B per position of the padded MB-grid frame (SURVEY §8(d): 1 B read "
                                          "+ 15 B written)",
                          "limiter": "issue / latency, not HBM (ncu: the planes land in L2; DESIGN.md §6)",
