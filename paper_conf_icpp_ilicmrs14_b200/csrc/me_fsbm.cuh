@@ -403,7 +403,10 @@ __global__ void __launch_bounds__(S_CT ? 128 : 256, S_CT ? FEVES_ME_MINB : 2) me
   // Small SAs (S <= 32: one RF window of few candidates per CTA, latency-bound grids) keep the
   // CF word in a register and store it after the first window's loads are issued, so the two
   // global round trips overlap instead of serialising (the S = 64 / 128 kernels are unchanged).
-  constexpr bool kLateCf = S_CT > 0 && S_CT <= 32 && !FUSE;
+#ifndef FEVES_ME_LATECF_MAX
+#define FEVES_ME_LATECF_MAX 32
+#endif
+  constexpr bool kLateCf = S_CT > 0 && S_CT <= FEVES_ME_LATECF_MAX && !FUSE;
   uint32_t cf_w[2] = {0, 0};                              // 64 words over 32 (S = 32) or 64 (S = 16) threads
   if (kLateCf) {
 #pragma unroll
