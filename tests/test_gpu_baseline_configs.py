@@ -97,11 +97,12 @@ def config3(orc):
     return cfg, frames, _oracle_frames(orc, frames, cfg.n_rf, cfg.sa_range)
 
 
-@pytest.mark.parametrize("host,graph", [(True, False), (False, False), (False, True)])
+@pytest.mark.parametrize("host,graph", [(True, False), (True, True), (False, False), (False, True)])
 def test_config3_1080p_s64_4rf_stream_every_mb(feves, config3, host, graph):
     """BASELINE config 3 (the bench workload): 1080p, 4 RFs, SA 64x64, INT || ME -> SME through
-    me_stream_push (host buffers = bench e2e; device buffers, captured as CUDA graphs = bench
-    value), 6 frames (RF ramp 1, 2, 3, 4, 4), every MB of every frame == oracle."""
+    me_stream_push (host buffers = bench e2e, with ME_OPT_GRAPH set too -- it applies to device
+    pushes only; device buffers, captured as CUDA graphs = bench value), 6 frames (RF ramp 1, 2, 3,
+    4, 4), every MB of every frame == oracle."""
     cfg, frames, ref = config3
     _compare(_push_all(feves, cfg, frames, host, graph=graph), ref, cfg.n_rf)
 

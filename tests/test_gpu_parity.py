@@ -352,12 +352,15 @@ def test_stream_push_host_buffers(feves, orc):
     me.close()
 
 
-def test_stream_host_pipeline_many_frames(feves, orc):
-    """host pushes back to back (uploads/downloads overlap compute on copy streams):
-    every frame's host outputs, captured into its own pinned buffer, match the oracle"""
+@pytest.mark.parametrize("graph", [0, 1])
+def test_stream_host_pipeline_many_frames(feves, orc, graph):
+    """host pushes back to back (uploads/downloads overlap compute on copy streams), with
+    ME_OPT_GRAPH off and on (host pushes are never captured): every frame's host outputs,
+    captured into its own pinned buffer, match the oracle"""
     W, H, S, n_rf = 64, 48, 8, 2
-    frames = [gen_tex(W, H, t, 23) for t in range(7)]
+    frames = [gen_tex(W, H, t, 23) for t in range(11)]
     me = feves.MotionEstimator(W, H, S, n_rf)
+    me.set_option(me.OPT_GRAPH, graph)
     n = me.mb_rows * me.mb_cols
     outs = []
     for f in frames:
