@@ -322,3 +322,20 @@ def test_sme_split_modes(feves, orc, split):
     np.testing.assert_array_equal(qs.cpu().numpy().reshape(n, 2, 41), o_qs)
     np.testing.assert_array_equal(q.cpu().numpy().reshape(n, 2, 41, 2), o_q)
     me.close()
+
+
+def test_scheduling_option_values(feves):
+    """ME_OPT_RF_PER_CTA accepts -1 (auto) .. 16, ME_OPT_SME_SPLIT 0 .. 3; anything else is
+    ME_EINVAL and leaves the context usable"""
+    me = feves.MotionEstimator(32, 32, 16, 2)
+    for v in (-1, 0, 1, 16):
+        me.set_option(me.OPT_RF_PER_CTA, v)
+    for v in (0, 1, 2, 3):
+        me.set_option(me.OPT_SME_SPLIT, v)
+    for opt, bad in ((me.OPT_RF_PER_CTA, -2), (me.OPT_RF_PER_CTA, 17), (me.OPT_SME_SPLIT, -1), (me.OPT_SME_SPLIT, 4)):
+        with pytest.raises(feves.FevesError):
+            me.set_option(opt, bad)
+    f = _dev(gen_tex(32, 32, 1, 2))
+    me.estimate(f, [f, f])                    # still usable
+    torch.cuda.synchronize()
+    me.close()
