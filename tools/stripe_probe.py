@@ -27,9 +27,11 @@ for n, rpc, spl in [(int(a), r, p) for a in (sys.argv[1:] or ["1", "2", "4", "8"
     me = F.MotionEstimator(cfg.width, cfg.height, cfg.sa_range, cfg.n_rf)
     me.set_option(me.OPT_RF_PER_CTA, rpc)
     me.set_option(me.OPT_SME_SPLIT, spl)
+    if os.environ.get("PIPE"):
+        me.set_option(me.OPT_PIPELINE_RF, int(os.environ["PIPE"]))
     r0, r1 = stripes(me.mb_rows, n)[0]                  # the largest stripe (first ranks get the extra row)
     me.set_rows(r0, r1)
-    me.set_option(me.OPT_GRAPH, 1)
+    me.set_option(me.OPT_GRAPH, int(os.environ.get("GRAPH", "1")))
     if n > 1:
         me.set_option(me.OPT_HALO_ONLY, 1)
     out = (torch.empty(me.mv_shape() + (2,), dtype=torch.int16, device="cuda"),
