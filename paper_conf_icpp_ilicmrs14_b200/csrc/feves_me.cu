@@ -475,9 +475,9 @@ static int launch_me(me_ctx* c, const uint8_t* cf, const uint8_t* const* rfs, in
   // RFs per CTA (ME_OPT_RF_PER_CTA, default 1: one CTA per (MB, RF)): more, shorter CTAs
   // desynchronise their window stagings across waves and shorten the last wave -- the frame and,
   // more so, a narrow MB-row stripe of a multi-GPU split
-  int rpc = n_ref;
+  int rpc = std::max(1, n_ref);
   const int want = c->rf_per_cta < 0 ? (c->S >= 128 ? 2 : 1) : c->rf_per_cta;
-  if (!fused && want > 0) rpc = std::min(n_ref, want);
+  if (!fused && want > 0) rpc = std::max(1, std::min(n_ref, want));
   P.rf_per_cta = rpc;
   dim3 grid(c->mb_cols, c->row1 - c->row0, (n_ref + rpc - 1) / rpc);
   size_t smem = fused ? c->me_smem_fused : c->me_smem;
