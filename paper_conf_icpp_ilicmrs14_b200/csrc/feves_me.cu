@@ -450,6 +450,7 @@ static void tmark(me_ctx* c, int i, cudaStream_t st) {
 static int launch_me(me_ctx* c, const uint8_t* cf, const uint8_t* const* rfs, int16_t* mvs, uint16_t* sads,
                      int n_ref, cudaStream_t st, const uint8_t* const* sfs = nullptr, int16_t* qmvs = nullptr,
                      uint16_t* qsads = nullptr, int rf0 = 0) {
+  if (n_ref <= 0) return ME_OK;   // nothing to search (the kernel would write nothing)
   MeParams P;
   memset(&P, 0, sizeof(P));
   P.cf = cf;
