@@ -428,7 +428,7 @@ __device__ __forceinline__ void refine_mode(const SmeParams& P, const uint8_t* _
 }
 
 #ifndef FEVES_SME_MINB
-#define FEVES_SME_MINB 5   // 96 registers, 5 CTAs x 4 warps per SM; with 32-bit row offsets (FEVES_SME_OFF32) 8 B of stack, 1 spill + 3 reloads per partition group outside the sweeps (was 72 B / 56 sites at 80 registers); 4 (128 registers): none, 147.5 vs 145.4 us; 5 / 6: 145.4 us
+#define FEVES_SME_MINB 5   // 96 registers, 5 CTAs x 4 warps per SM; with 32-bit row offsets (FEVES_SME_OFF32) 8 B of stack, 1 spill + 3 reloads per partition group outside the sweeps (was 72 B / 56 sites at 80 registers); 4 (128 registers): none, 147.5 vs 145.4 us; 5 / 6: 145.4 us; with the longest-first order 6 (80 registers, 16 B stack, 10 spill sites) 139.7 vs 141.4 us -- kept 5 (spill-free sweeps)
 #endif
 template <bool RD, bool SATD>
 __global__ void __launch_bounds__(128, FEVES_SME_MINB) sme_refine_kernel(const SmeParams P) {
